@@ -1,0 +1,205 @@
+"""The CPU oracle for the G1 MSM — TEST INFRASTRUCTURE ONLY.
+
+Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline and
+``--impl reference`` legs may import this package.  The product package
+(paper_conf_asplos_maxsm0k0zsh23_b200) never imports it, and it never imports
+the product: the two share no code.
+
+Two independent oracles live here:
+
+* ``oracle.ref``  — Python ints, affine chord-and-tangent, double-and-add
+  (tiny inputs; cross-checks the C oracle);
+* ``liboracle.so`` (oracle.c) — the same definition in plain C with
+  schoolbook bignums and Knuth-D remainders, threaded over the host cores.
+
+Both compute the definition Q = sum_i k_i (x) P_i (§2.1).
+Pins: tests/test_oracle_pins.py.
+"""
+
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+from . import curves, ref
+from .curves import Curve, get
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_SRC = os.path.join(_HERE, "oracle.c")
+_lib = None
+
+
+def build(force: bool = False) -> str:
+    """Compile oracle.c with gcc (plain -O2, no vectorisation tricks)."""
+    if force or not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(_SRC):
+        tmp = _SO + ".tmp.%d" % os.getpid()
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-shared", "-fPIC", "-pthread",
+                               _SRC, "-o", tmp])
+        os.replace(tmp, _SO)
+    return _SO
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(_SO)
+        u32p = ctypes.POINTER(ctypes.c_uint32)
+        for name, args in {
+            "oracle_msm": [ctypes.c_int, u32p, u32p, u32p, u32p, ctypes.c_int, ctypes.c_uint64, u32p, ctypes.c_int],
+            "oracle_mul_each": [ctypes.c_int, u32p, u32p, u32p, u32p, ctypes.c_int, ctypes.c_uint64, u32p, ctypes.c_int],
+            "oracle_ec_add": [ctypes.c_int, u32p, u32p, u32p, u32p, u32p],
+            "oracle_fp_mul": [ctypes.c_int, u32p, u32p, u32p, u32p],
+            "oracle_fp_inv": [ctypes.c_int, u32p, u32p, u32p],
+            "oracle_bn_mod": [u32p, ctypes.c_int, u32p, ctypes.c_int, u32p],
+        }.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def default_threads() -> int:
+    try:
+        return max(1, len(os.sched_getaffinity(0)))
+    except AttributeError:
+        return os.cpu_count() or 1
+
+
+def _p(a: np.ndarray):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_uint32))
+
+
+def _u32(a) -> np.ndarray:
+    return np.ascontiguousarray(a, dtype=np.uint32)
+
+
+def _consts(c: Curve):
+    L = c.limbs
+    return L, _u32(ref.int_to_limbs(c.p, L)), _u32(ref.int_to_limbs(c.a % c.p, L))
+
+
+def msm(curve, points: np.ndarray, scalars: np.ndarray, nthreads: int | None = None) -> np.ndarray:
+    """C oracle MSM.  points: [n, 2L] u32 canonical affine ((0,0) = O);
+    scalars: [n, Ls] u32 little-endian.  Returns [2L] u32 (affine, (0,0) = O)."""
+    c = get(curve)
+    L, p, a = _consts(c)
+    points = _u32(points).reshape(-1, 2 * L)
+    scalars = _u32(scalars)
+    n = points.shape[0]
+    Ls = scalars.shape[1] if scalars.ndim == 2 else 1
+    scalars = scalars.reshape(n, Ls)
+    out = np.zeros(2 * L, dtype=np.uint32)
+    rc = lib().oracle_msm(L, _p(p), _p(a), _p(points), _p(scalars), Ls, n, _p(out),
+                          nthreads or default_threads())
+    if rc:
+        raise RuntimeError(f"oracle_msm failed: {rc}")
+    return out
+
+
+def mul_each(curve, P: np.ndarray, scalars: np.ndarray, nthreads: int | None = None) -> np.ndarray:
+    """out[i] = k_i (x) P (C oracle).  Returns [n, 2L] u32."""
+    c = get(curve)
+    L, p, a = _consts(c)
+    P = _u32(P).reshape(2 * L)
+    scalars = _u32(scalars)
+    n = scalars.shape[0]
+    Ls = scalars.shape[1] if scalars.ndim == 2 else 1
+    scalars = scalars.reshape(n, Ls)
+    out = np.zeros((n, 2 * L), dtype=np.uint32)
+    rc = lib().oracle_mul_each(L, _p(p), _p(a), _p(P), _p(scalars), Ls, n, _p(out),
+                               nthreads or default_threads())
+    if rc:
+        raise RuntimeError(f"oracle_mul_each failed: {rc}")
+    return out
+
+
+def generator_limbs(curve) -> np.ndarray:
+    c = get(curve)
+    return _u32(ref.encode_point(c, (c.gx, c.gy)))
+
+
+def points_from_dlogs(curve, dlogs: np.ndarray, nthreads: int | None = None) -> np.ndarray:
+    """P_i = a_i (x) G, the synthetic proving-key points with known discrete
+    logs (SURVEY.md §8(d) "Points")."""
+    return mul_each(curve, generator_limbs(curve), dlogs, nthreads)
+
+
+def ec_add(curve, P: np.ndarray, Q: np.ndarray) -> np.ndarray:
+    c = get(curve)
+    L, p, a = _consts(c)
+    out = np.zeros(2 * L, dtype=np.uint32)
+    rc = lib().oracle_ec_add(L, _p(p), _p(a), _p(_u32(P)), _p(_u32(Q)), _p(out))
+    if rc:
+        raise RuntimeError(f"oracle_ec_add failed: {rc}")
+    return out
+
+
+def fp_mul(curve, x: int, y: int) -> int:
+    c = get(curve)
+    L, p, _ = _consts(c)
+    out = np.zeros(L, dtype=np.uint32)
+    X, Y = _u32(ref.int_to_limbs(x, L)), _u32(ref.int_to_limbs(y, L))
+    if lib().oracle_fp_mul(L, _p(p), _p(X), _p(Y), _p(out)):
+        raise RuntimeError("oracle_fp_mul failed")
+    return ref.limbs_to_int(out)
+
+
+def fp_inv(curve, x: int) -> int:
+    c = get(curve)
+    L, p, _ = _consts(c)
+    out = np.zeros(L, dtype=np.uint32)
+    X = _u32(ref.int_to_limbs(x, L))
+    if lib().oracle_fp_inv(L, _p(p), _p(X), _p(out)):
+        raise RuntimeError("oracle_fp_inv failed")
+    return ref.limbs_to_int(out)
+
+
+def bn_mod(u: int, m: int, v: int, n: int) -> int:
+    U = _u32(ref.int_to_limbs(u, m))
+    V = _u32(ref.int_to_limbs(v, n))
+    out = np.zeros(n, dtype=np.uint32)
+    if lib().oracle_bn_mod(_p(U), m, _p(V), n, _p(out)):
+        raise RuntimeError("oracle_bn_mod failed")
+    return ref.limbs_to_int(out)
+
+
+def closed_form(curve, scalars: np.ndarray, dlogs: np.ndarray) -> np.ndarray:
+    """sum_i k_i (a_i G) = (sum_i k_i a_i mod r) G  (SURVEY.md §8(c) pins).
+
+    The exact integer sum_i k_i a_i is computed with 16-bit limbs so that every
+    numpy partial sum stays below 2^64 (each product < 2^32, n < 2^31)."""
+    c = get(curve)
+    s = dot_mod(scalars, dlogs, c.r)
+    Ls = c.scalar_limbs
+    k = _u32(ref.int_to_limbs(s, Ls)).reshape(1, Ls)
+    return mul_each(c, generator_limbs(c), k, 1)[0]
+
+
+def dot_mod(scalars: np.ndarray, dlogs: np.ndarray, r: int) -> int:
+    """(sum_i k_i a_i) mod r, exactly, for u32-limb arrays."""
+    k16 = _u32(scalars).view(np.uint16).astype(np.uint64)   # little-endian halves
+    a16 = _u32(dlogs).view(np.uint16).astype(np.uint64)
+    n = k16.shape[0]
+    if n >= (1 << 31):
+        raise ValueError("n too large for exact 16-bit accumulation")
+    total = 0
+    # M[u, v] = sum_i k16[i,u] * a16[i,v]  (exact in uint64)
+    step = 1 << 20
+    for s0 in range(0, n, step):
+        M = k16[s0:s0 + step].T @ a16[s0:s0 + step]
+        for u in range(M.shape[0]):
+            for v in range(M.shape[1]):
+                m = int(M[u, v])
+                if m:
+                    total += m << (16 * (u + v))
+    return total % r
+
+
+__all__ = ["curves", "ref", "msm", "mul_each", "points_from_dlogs", "closed_form", "dot_mod",
+           "ec_add", "fp_mul", "fp_inv", "bn_mod", "build", "default_threads", "generator_limbs"]

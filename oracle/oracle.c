@@ -1,0 +1,435 @@
+/*
+ * oracle.c -- plain, slow CPU reference for the G1 MSM.
+ *
+ *   TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and
+ *   bench.py's cpu_baseline / --impl reference legs may load this library.
+ *   It shares no code, header, table or constant with the CUDA product path
+ *   (paper_conf_asplos_maxsm0k0zsh23_b200/csrc); curve constants are passed
+ *   in by the caller (oracle/curves.py holds the oracle's own copy).
+ *
+ * What it computes is the definition (§2.1):
+ *     Q = sum_{i<n} k_i (x) P_i      over E(F_p): y^2 = x^3 + a x + b
+ *
+ *   1. bignum: u32 limbs, schoolbook products, remainder by Knuth's
+ *      Algorithm D (TAOCP 4.3.1).  No Montgomery form.
+ *   2. field inverse: the binary extended Euclidean algorithm (HAC 14.61,
+ *      specialised to an odd modulus).
+ *   3. group law: AFFINE chord-and-tangent formulas with every exceptional
+ *      case explicit (O, P == Q, P == -Q); "PADD ... including point doubling"
+ *      (PAPER.md:116 fn. 2).
+ *   4. PMUL: left-to-right binary double-and-add.
+ *   5. MSM: each thread sums k_i P_i over a contiguous chunk; the chunk sums
+ *      are added in chunk order.  The group is abelian and exact, so the
+ *      result is independent of the order.
+ *
+ * Encoding: a point is 2L little-endian u32 limbs x || y, canonical (< p);
+ * the identity O is (0,0).  A scalar is Ls little-endian u32 limbs, any
+ * integer (not reduced mod r).
+ */
+#include <pthread.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+#define MAXL 24
+
+typedef struct {
+    int L;               /* limbs of the encoding */
+    int Le;              /* effective limbs of p (top limb nonzero) */
+    uint32_t p[MAXL];
+    uint32_t a[MAXL];
+} fctx;
+
+typedef struct {
+    uint32_t x[MAXL], y[MAXL];
+    int inf;             /* 1 = identity O */
+} apt;
+
+/* ------------------------------------------------------------------ bignum */
+
+static int bn_cmp(const uint32_t *x, const uint32_t *y, int n) {
+    for (int i = n - 1; i >= 0; --i) {
+        if (x[i] != y[i]) return x[i] > y[i] ? 1 : -1;
+    }
+    return 0;
+}
+
+static int bn_is_zero(const uint32_t *x, int n) {
+    for (int i = 0; i < n; ++i)
+        if (x[i]) return 0;
+    return 1;
+}
+
+static int bn_is_one(const uint32_t *x, int n) {
+    if (x[0] != 1) return 0;
+    for (int i = 1; i < n; ++i)
+        if (x[i]) return 0;
+    return 1;
+}
+
+static uint32_t bn_add(uint32_t *r, const uint32_t *x, const uint32_t *y, int n) {
+    uint64_t c = 0;
+    for (int i = 0; i < n; ++i) {
+        c += (uint64_t)x[i] + y[i];
+        r[i] = (uint32_t)c;
+        c >>= 32;
+    }
+    return (uint32_t)c;
+}
+
+static uint32_t bn_sub(uint32_t *r, const uint32_t *x, const uint32_t *y, int n) {
+    int64_t b = 0;
+    for (int i = 0; i < n; ++i) {
+        int64_t t = (int64_t)x[i] - y[i] + b;
+        r[i] = (uint32_t)t;
+        b = t >> 32;            /* 0 or -1 */
+    }
+    return (uint32_t)(b & 1);
+}
+
+/* x >>= 1, shifting `top` in as the new most significant bit */
+static void bn_shr1(uint32_t *x, int n, uint32_t top) {
+    for (int i = 0; i < n - 1; ++i) x[i] = (x[i] >> 1) | (x[i + 1] << 31);
+    x[n - 1] = (x[n - 1] >> 1) | (top << 31);
+}
+
+/* schoolbook product: t[0..2n) = x * y */
+static void bn_mul(uint32_t *t, const uint32_t *x, const uint32_t *y, int n) {
+    memset(t, 0, sizeof(uint32_t) * 2 * n);
+    for (int i = 0; i < n; ++i) {
+        uint64_t c = 0;
+        for (int j = 0; j < n; ++j) {
+            c += (uint64_t)x[i] * y[j] + t[i + j];
+            t[i + j] = (uint32_t)c;
+            c >>= 32;
+        }
+        t[i + n] = (uint32_t)c;
+    }
+}
+
+/* Knuth Algorithm D remainder: r[0..n) = u[0..m) mod v[0..n), v[n-1] != 0, m >= n */
+static void bn_mod(uint32_t *r, const uint32_t *u, int m, const uint32_t *v, int n) {
+    if (n == 1) {
+        uint64_t rem = 0;
+        for (int i = m - 1; i >= 0; --i) rem = ((rem << 32) | u[i]) % v[0];
+        r[0] = (uint32_t)rem;
+        return;
+    }
+    uint32_t un[2 * MAXL + 1], vn[MAXL];
+    int s = __builtin_clz(v[n - 1]);
+    for (int i = n - 1; i > 0; --i)
+        vn[i] = (v[i] << s) | (s ? (uint32_t)((uint64_t)v[i - 1] >> (32 - s)) : 0);
+    vn[0] = v[0] << s;
+    un[m] = s ? (uint32_t)((uint64_t)u[m - 1] >> (32 - s)) : 0;
+    for (int i = m - 1; i > 0; --i)
+        un[i] = (u[i] << s) | (s ? (uint32_t)((uint64_t)u[i - 1] >> (32 - s)) : 0);
+    un[0] = u[0] << s;
+
+    const uint64_t B = 1ull << 32;
+    for (int j = m - n; j >= 0; --j) {
+        uint64_t num = ((uint64_t)un[j + n] << 32) | un[j + n - 1];
+        uint64_t qhat = num / vn[n - 1];
+        uint64_t rhat = num % vn[n - 1];
+        while (qhat >= B || qhat * vn[n - 2] > ((rhat << 32) | un[j + n - 2])) {
+            qhat--;
+            rhat += vn[n - 1];
+            if (rhat >= B) break;
+        }
+        /* multiply and subtract */
+        int64_t borrow = 0;
+        uint64_t carry = 0;
+        for (int i = 0; i < n; ++i) {
+            uint64_t prod = qhat * vn[i] + carry;
+            carry = prod >> 32;
+            int64_t t = (int64_t)un[i + j] - (int64_t)(uint32_t)prod + borrow;
+            un[i + j] = (uint32_t)t;
+            borrow = t >> 32;
+        }
+        int64_t t = (int64_t)un[j + n] - (int64_t)carry + borrow;
+        un[j + n] = (uint32_t)t;
+        if (t < 0) {            /* qhat was one too large: add v back */
+            uint64_t c = 0;
+            for (int i = 0; i < n; ++i) {
+                c += (uint64_t)un[i + j] + vn[i];
+                un[i + j] = (uint32_t)c;
+                c >>= 32;
+            }
+            un[j + n] += (uint32_t)c;
+        }
+    }
+    for (int i = 0; i < n; ++i)
+        r[i] = (un[i] >> s) | (s ? (uint32_t)((uint64_t)un[i + 1] << (32 - s)) : 0);
+}
+
+/* ------------------------------------------------------------------- F_p */
+
+static void fp_add(const fctx *f, uint32_t *r, const uint32_t *x, const uint32_t *y) {
+    uint32_t t[MAXL];
+    uint32_t c = bn_add(t, x, y, f->L);
+    if (c || bn_cmp(t, f->p, f->L) >= 0) bn_sub(t, t, f->p, f->L);
+    memcpy(r, t, sizeof(uint32_t) * f->L);
+}
+
+static void fp_sub(const fctx *f, uint32_t *r, const uint32_t *x, const uint32_t *y) {
+    uint32_t t[MAXL];
+    if (bn_sub(t, x, y, f->L)) bn_add(t, t, f->p, f->L);
+    memcpy(r, t, sizeof(uint32_t) * f->L);
+}
+
+static void fp_mul(const fctx *f, uint32_t *r, const uint32_t *x, const uint32_t *y) {
+    uint32_t t[2 * MAXL], q[MAXL];
+    bn_mul(t, x, y, f->L);
+    memset(q, 0, sizeof(q));
+    bn_mod(q, t, 2 * f->L, f->p, f->Le);
+    memcpy(r, q, sizeof(uint32_t) * f->L);
+}
+
+/* (x + p) / 2 or x / 2 modulo p, for x in [0, p) */
+static void fp_half(const fctx *f, uint32_t *x) {
+    if (x[0] & 1) {
+        uint32_t c = bn_add(x, x, f->p, f->L);
+        bn_shr1(x, f->L, c);
+    } else {
+        bn_shr1(x, f->L, 0);
+    }
+}
+
+/* binary extended Euclid (HAC 14.61 for odd p); x != 0 required */
+static void fp_inv(const fctx *f, uint32_t *r, const uint32_t *x) {
+    int L = f->L;
+    uint32_t u[MAXL], v[MAXL], x1[MAXL], x2[MAXL];
+    memcpy(u, x, sizeof(uint32_t) * L);
+    memcpy(v, f->p, sizeof(uint32_t) * L);
+    memset(x1, 0, sizeof(x1));
+    memset(x2, 0, sizeof(x2));
+    x1[0] = 1;
+    while (!bn_is_one(u, L) && !bn_is_one(v, L)) {
+        while (!(u[0] & 1)) { bn_shr1(u, L, 0); fp_half(f, x1); }
+        while (!(v[0] & 1)) { bn_shr1(v, L, 0); fp_half(f, x2); }
+        if (bn_cmp(u, v, L) >= 0) {
+            bn_sub(u, u, v, L);
+            fp_sub(f, x1, x1, x2);
+        } else {
+            bn_sub(v, v, u, L);
+            fp_sub(f, x2, x2, x1);
+        }
+    }
+    memcpy(r, bn_is_one(u, L) ? x1 : x2, sizeof(uint32_t) * L);
+}
+
+/* ------------------------------------------------------------ group law */
+
+static void ec_add(const fctx *f, apt *R, const apt *P, const apt *Q) {
+    int L = f->L;
+    if (P->inf) { *R = *Q; return; }
+    if (Q->inf) { *R = *P; return; }
+    uint32_t lam[MAXL], num[MAXL], den[MAXL], t[MAXL];
+    if (bn_cmp(P->x, Q->x, L) == 0) {
+        fp_add(f, t, P->y, Q->y);
+        if (bn_is_zero(t, L)) {             /* P == -Q */
+            memset(R, 0, sizeof(*R));
+            R->inf = 1;
+            return;
+        }
+        /* tangent: lam = (3 x^2 + a) / (2 y) */
+        fp_mul(f, t, P->x, P->x);
+        fp_add(f, num, t, t);
+        fp_add(f, num, num, t);
+        fp_add(f, num, num, f->a);
+        fp_add(f, den, P->y, P->y);
+    } else {
+        /* chord: lam = (y2 - y1) / (x2 - x1) */
+        fp_sub(f, num, Q->y, P->y);
+        fp_sub(f, den, Q->x, P->x);
+    }
+    fp_inv(f, t, den);
+    fp_mul(f, lam, num, t);
+    uint32_t x3[MAXL], y3[MAXL];
+    fp_mul(f, x3, lam, lam);
+    fp_sub(f, x3, x3, P->x);
+    fp_sub(f, x3, x3, Q->x);
+    fp_sub(f, t, P->x, x3);
+    fp_mul(f, y3, lam, t);
+    fp_sub(f, y3, y3, P->y);
+    memset(R, 0, sizeof(*R));
+    memcpy(R->x, x3, sizeof(uint32_t) * L);
+    memcpy(R->y, y3, sizeof(uint32_t) * L);
+    R->inf = 0;
+}
+
+/* left-to-right double-and-add over the Ls-limb scalar k */
+static void ec_mul(const fctx *f, apt *R, const uint32_t *k, int Ls, const apt *P) {
+    apt acc;
+    memset(&acc, 0, sizeof(acc));
+    acc.inf = 1;
+    for (int i = 32 * Ls - 1; i >= 0; --i) {
+        apt t;
+        ec_add(f, &t, &acc, &acc);
+        acc = t;
+        if ((k[i / 32] >> (i % 32)) & 1) {
+            ec_add(f, &t, &acc, P);
+            acc = t;
+        }
+    }
+    *R = acc;
+}
+
+static void load_point(const fctx *f, apt *P, const uint32_t *src) {
+    memset(P, 0, sizeof(*P));
+    memcpy(P->x, src, sizeof(uint32_t) * f->L);
+    memcpy(P->y, src + f->L, sizeof(uint32_t) * f->L);
+    P->inf = bn_is_zero(P->x, f->L) && bn_is_zero(P->y, f->L);
+}
+
+static void store_point(const fctx *f, uint32_t *dst, const apt *P) {
+    if (P->inf) {
+        memset(dst, 0, sizeof(uint32_t) * 2 * f->L);
+        return;
+    }
+    memcpy(dst, P->x, sizeof(uint32_t) * f->L);
+    memcpy(dst + f->L, P->y, sizeof(uint32_t) * f->L);
+}
+
+static int init_ctx(fctx *f, int L, const uint32_t *p, const uint32_t *a) {
+    if (L < 1 || L > MAXL) return -1;
+    memset(f, 0, sizeof(*f));
+    f->L = L;
+    memcpy(f->p, p, sizeof(uint32_t) * L);
+    memcpy(f->a, a, sizeof(uint32_t) * L);
+    f->Le = L;
+    while (f->Le > 1 && f->p[f->Le - 1] == 0) f->Le--;
+    if (!(f->p[0] & 1)) return -1;
+    return 0;
+}
+
+/* ------------------------------------------------------------- threading */
+
+typedef struct {
+    const fctx *f;
+    const uint32_t *points, *scalars;
+    int Ls;
+    uint64_t begin, end;
+    uint32_t *out;         /* msm: one point; mul_each: n points */
+    int each;
+} job;
+
+static void *run_job(void *arg) {
+    job *j = (job *)arg;
+    const fctx *f = j->f;
+    apt acc;
+    memset(&acc, 0, sizeof(acc));
+    acc.inf = 1;
+    for (uint64_t i = j->begin; i < j->end; ++i) {
+        apt P, R;
+        const uint32_t *k = j->scalars + (size_t)i * j->Ls;
+        load_point(f, &P, j->points + (j->each ? 0 : (size_t)i * 2 * f->L));
+        if (P.inf || bn_is_zero(k, j->Ls)) {
+            memset(&R, 0, sizeof(R));
+            R.inf = 1;
+        } else {
+            ec_mul(f, &R, k, j->Ls, &P);
+        }
+        if (j->each) {
+            store_point(f, j->out + (size_t)i * 2 * f->L, &R);
+        } else {
+            apt t;
+            ec_add(f, &t, &acc, &R);
+            acc = t;
+        }
+    }
+    if (!j->each) store_point(f, j->out, &acc);
+    return NULL;
+}
+
+static int run_parallel(const fctx *f, const uint32_t *points, const uint32_t *scalars, int Ls,
+                        uint64_t n, uint32_t *out, int nthreads, int each) {
+    if (nthreads < 1) nthreads = 1;
+    if ((uint64_t)nthreads > n) nthreads = n ? (int)n : 1;
+    job *jobs = (job *)calloc(nthreads, sizeof(job));
+    pthread_t *th = (pthread_t *)calloc(nthreads, sizeof(pthread_t));
+    uint32_t *partial = (uint32_t *)calloc((size_t)nthreads * 2 * f->L, sizeof(uint32_t));
+    if (!jobs || !th || !partial) { free(jobs); free(th); free(partial); return -2; }
+    uint64_t chunk = (n + nthreads - 1) / nthreads;
+    for (int t = 0; t < nthreads; ++t) {
+        jobs[t].f = f;
+        jobs[t].points = points;
+        jobs[t].scalars = scalars;
+        jobs[t].Ls = Ls;
+        jobs[t].begin = (uint64_t)t * chunk < n ? (uint64_t)t * chunk : n;
+        jobs[t].end = (uint64_t)(t + 1) * chunk < n ? (uint64_t)(t + 1) * chunk : n;
+        jobs[t].out = each ? out : partial + (size_t)t * 2 * f->L;
+        jobs[t].each = each;
+        pthread_create(&th[t], NULL, run_job, &jobs[t]);
+    }
+    for (int t = 0; t < nthreads; ++t) pthread_join(th[t], NULL);
+    if (!each) {
+        apt acc, P, s;
+        memset(&acc, 0, sizeof(acc));
+        acc.inf = 1;
+        for (int t = 0; t < nthreads; ++t) {
+            load_point(f, &P, partial + (size_t)t * 2 * f->L);
+            ec_add(f, &s, &acc, &P);
+            acc = s;
+        }
+        store_point(f, out, &acc);
+    }
+    free(jobs);
+    free(th);
+    free(partial);
+    return 0;
+}
+
+/* ------------------------------------------------------------- exports */
+
+/* Q = sum k_i P_i.  points: n x 2L limbs; scalars: n x Ls limbs; out: 2L limbs. */
+int oracle_msm(int L, const uint32_t *p, const uint32_t *a, const uint32_t *points,
+               const uint32_t *scalars, int Ls, uint64_t n, uint32_t *out, int nthreads) {
+    fctx f;
+    if (init_ctx(&f, L, p, a)) return -1;
+    return run_parallel(&f, points, scalars, Ls, n, out, nthreads, 0);
+}
+
+/* out_i = k_i P for one base point P (2L limbs); out: n x 2L limbs. */
+int oracle_mul_each(int L, const uint32_t *p, const uint32_t *a, const uint32_t *P,
+                    const uint32_t *scalars, int Ls, uint64_t n, uint32_t *out, int nthreads) {
+    fctx f;
+    if (init_ctx(&f, L, p, a)) return -1;
+    return run_parallel(&f, P, scalars, Ls, n, out, nthreads, 1);
+}
+
+/* R = P + Q (affine, explicit cases) */
+int oracle_ec_add(int L, const uint32_t *p, const uint32_t *a, const uint32_t *P,
+                  const uint32_t *Q, uint32_t *R) {
+    fctx f;
+    if (init_ctx(&f, L, p, a)) return -1;
+    apt A, B, C;
+    load_point(&f, &A, P);
+    load_point(&f, &B, Q);
+    ec_add(&f, &C, &A, &B);
+    store_point(&f, R, &C);
+    return 0;
+}
+
+int oracle_fp_mul(int L, const uint32_t *p, const uint32_t *x, const uint32_t *y, uint32_t *r) {
+    fctx f;
+    uint32_t zero[MAXL] = {0};
+    if (init_ctx(&f, L, p, zero)) return -1;
+    fp_mul(&f, r, x, y);
+    return 0;
+}
+
+int oracle_fp_inv(int L, const uint32_t *p, const uint32_t *x, uint32_t *r) {
+    fctx f;
+    uint32_t zero[MAXL] = {0};
+    if (init_ctx(&f, L, p, zero)) return -1;
+    if (bn_is_zero(x, L)) return -3;
+    fp_inv(&f, r, x);
+    return 0;
+}
+
+/* r = u mod v (Knuth D), exported so the tests can pin it against Python ints */
+int oracle_bn_mod(const uint32_t *u, int m, const uint32_t *v, int n, uint32_t *r) {
+    if (n < 1 || n > MAXL || m < n || m > 2 * MAXL || v[n - 1] == 0) return -1;
+    bn_mod(r, u, m, v, n);
+    return 0;
+}
