@@ -1,0 +1,395 @@
+#!/usr/bin/env python
+"""Benchmark: G1 MSM points/s on B200 (BASELINE.json metric), one JSON line.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--workload NAME] [--impl gzkp|reference]
+
+A "step" is one full MSM (all of SURVEY.md §8(a): digits, sort, bucket
+accumulation, merge, bucket reduction, window combination, normalisation)
+over the workload's n points.  Default workload: BLS12-381, n = 2^22, uniform
+scalars (BASELINE configs[2], the config the metric is quoted on at 1/2/4/8
+GPUs).  Multi-GPU (torchrun, one rank per GPU): strong scaling, each rank runs
+the full Pippenger on its contiguous shard and the partial sums meet in ONE
+NCCL all-gather (gzkp_msm_sharded).
+
+Inputs are synthetic and seeded (synth/): scalars uniform in [0, r), points
+a_i * G with a_i uniform (generated on the device by the product's fixed-base
+kernel).  `value` is n / device time with inputs resident in HBM; `e2e` adds the
+host->device copy of points and scalars and the device->host read of the result
+every step.  The oracle (oracle/) runs only in the cpu_baseline leg and in
+--impl reference.
+"""
+
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+WORKLOADS = {
+    # name: (curve, log2 n, config index for seeds, scalar distribution, BASELINE config text)
+    "bls12_381_2p22": ("bls12_381", 22, 3, "uniform", "BLS12-381 G1 MSM n=2^22, uniform scalars"),
+    "bn254_2p20": ("bn254", 20, 2, "uniform", "BN254 G1 MSM n=2^20, uniform 254-bit scalars"),
+    "mnt4_753_2p20": ("mnt4_753", 20, 4, "uniform", "MNT4-753 G1 MSM n=2^20"),
+    "bls12_381_2p26_sparse": ("bls12_381", 26, 5, "zcash_like", "BLS12-381 G1 MSM n=2^26, sparse/skewed scalars"),
+    "bls12_381_2p26": ("bls12_381", 26, 6, "uniform", "BLS12-381 G1 MSM n=2^26, uniform scalars"),
+    "bn254_2p10": ("bn254", 10, 1, "uniform", "BN254 G1 MSM n=2^10, uniform random scalars"),
+}
+L_BY_CURVE = {"bn254": 8, "bls12_381": 12, "mnt4_753": 24}
+METRIC = "G1 MSM points/sec"
+L2_BYTES = 126 * 1024 * 1024
+
+
+def madd_imad(L: int) -> int:
+    """Algorithmic IMAD count of one XYZZ mixed add:
+    madd = 8M + 2S with M = 4L^2 + L, S = 3L^2 + 2L."""
+    return 8 * (4 * L * L + L) + 2 * (3 * L * L + 2 * L)
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except Exception:
+        return {"sm_max_mhz": 1965.0, "hbm_gbs": 6650.0}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+        self.lines = []
+        self.thread = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+            return
+        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        if self.thread:
+            self.thread.join(timeout=2)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(smax), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+# ------------------------------------------------------------- oracle legs
+
+def oracle_time_sample(curve: str, n_s: int, seed_cfg: int, dist: str, budget_s: float):
+    """Time the oracle MSM on a bounded sample of the workload (host cores)."""
+    import oracle
+    cores = oracle.default_threads()
+    m = min(n_s, max(8, 16 * cores))
+    d = synth.dlogs(curve, m, synth.dlog_seed(curve))
+    pts = oracle.points_from_dlogs(curve, d)
+    reps = (n_s + m - 1) // m
+    pts = np.tile(pts, (reps, 1))[:n_s]
+    k = synth.scalars(curve, n_s, synth.scalar_seed(seed_cfg), dist)
+    t0 = time.perf_counter()
+    out = oracle.msm(curve, pts, k, nthreads=cores)
+    wall = time.perf_counter() - t0
+    return n_s / wall, wall, cores, pts, k, out
+
+
+def calibrate_oracle_n(curve: str, budget_s: float) -> int:
+    import oracle
+    cores = oracle.default_threads()
+    n_cal = max(cores, 8)
+    rate, wall, *_ = oracle_time_sample(curve, n_cal, 0, "uniform", 1.0)
+    return max(cores, int(rate * budget_s))
+
+
+def run_reference(args, wl):
+    world, rank, _ = dist_env()
+    curve, logn, cfg, dist, desc = WORKLOADS[wl]
+    if rank != 0:
+        return
+    import oracle
+    cores = oracle.default_threads()
+    per_step = max(2.0, 90.0 / (args.steps + args.warmup))
+    n_s = calibrate_oracle_n(curve, per_step)
+    for _ in range(args.warmup):
+        oracle_time_sample(curve, max(cores, n_s // 8), cfg, dist, per_step)
+    walls = []
+    for _ in range(args.steps):
+        _, wall, *_ = oracle_time_sample(curve, n_s, cfg, dist, per_step)
+        walls.append(wall)
+    value = n_s * len(walls) / sum(walls)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "points/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(walls) / len(walls),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32 (exact F_p)",
+        "data": "synthetic",
+        "config": {"workload": wl, "curve": curve, "n": 1 << logn, "scalars": dist, "baseline_config": desc},
+        "cpu_baseline": {"value": value, "unit": "points/s", "cores": cores, "kind": "oracle",
+                         "sample": f"first {n_s} scalars of the workload, points tiled from "
+                                   f"{min(n_s, max(8, 16 * cores))} oracle-generated a_i*G; "
+                                   f"affine double-and-add MSM (oracle.c)"},
+        "e2e": {"value": value, "unit": "points/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ---------------------------------------------------------------- GPU arm
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="gzkp", choices=["gzkp", "reference"])
+    ap.add_argument("--workload", default="bls12_381_2p22", choices=sorted(WORKLOADS))
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--window-bits", type=int, default=0)
+    ap.add_argument("--chunk", type=int, default=0)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+    wl = args.workload
+
+    if args.impl == "reference":
+        run_reference(args, wl)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_asplos_maxsm0k0zsh23_b200 as gz
+    from paper_conf_asplos_maxsm0k0zsh23_b200 import build as gbuild
+
+    world, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    gbuild.build()
+    gz.set_config(args.window_bits, args.chunk)
+
+    curve, logn, cfg, sdist, desc = WORKLOADS[wl]
+    n = 1 << logn
+    L = L_BY_CURVE[curve]
+    lo, hi = gz.shard_range(n, world, rank)
+    n_loc = hi - lo
+
+    # ---- inputs (seeded; points generated on the device) ----
+    dl = synth.dlogs(curve, n, synth.dlog_seed(curve))[lo:hi]
+    ks = synth.scalars(curve, n, synth.scalar_seed(cfg), sdist)[lo:hi]
+    P = torch.empty((n_loc, 2 * L), dtype=torch.int32, device="cuda")
+    step_gen = 1 << 20
+    for s0 in range(0, n_loc, step_gen):
+        gz.fixed_base_mul(curve, gz.to_device(dl[s0:s0 + step_gen]), out=P[s0:s0 + step_gen])
+    K = gz.to_device(ks)
+    out = torch.empty(2 * L, dtype=torch.int32, device="cuda")
+    torch.cuda.synchronize()
+    comm = gz.Comm(world, rank) if world > 1 else None
+    stream = torch.cuda.current_stream()
+
+    def step():
+        if comm is None:
+            gz.msm(curve, P, K, out=out)
+        else:
+            gz.msm_sharded(curve, P, K, comm, out=out)
+
+    input_bytes = n_loc * (2 * L + ks.shape[1]) * 4
+    flush_l2 = input_bytes < 2 * L2_BYTES
+    flush_buf = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device="cuda") if flush_l2 else None
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    gz.set_profiling(True)
+    gz.profile_read(reset=True)
+    sampler = ClockSampler(local)
+    sampler.start()
+    time.sleep(0.3)
+
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    if flush_l2:
+        # per-step events, L2 flushed between steps outside the timed windows
+        total_ms = 0.0
+        for _ in range(args.steps):
+            flush_buf.zero_()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            step()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            total_ms += e0.elapsed_time(e1)
+    else:
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        total_ms = e0.elapsed_time(e1)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks = sampler.stop()
+    prof = gz.profile_read(reset=True)
+    gz.set_profiling(False)
+
+    t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    total_ms = float(t.item())
+    ms_per_step = total_ms / args.steps
+    value = n / (ms_per_step / 1e3)
+
+    # ---- roofline of the dominant kernel (bucket accumulation, k_accum) ----
+    peaks, peaks_src = load_peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    calls = max(1, prof["calls"])
+    accum_ms = prof["phase_ms"]["accumulate"] / calls
+    entries = prof["entries"]
+    imad_per_launch = entries * madd_imad(L)
+    achieved = imad_per_launch / (accum_ms / 1e3) if accum_ms > 0 else 0.0
+    peak = 148 * 64 * sm_max * 1e6
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "accum_traffic.json")) as f:
+            traffic = json.load(f).get(wl)
+    except Exception:
+        pass
+    phase_share = {k: round(v / calls, 4) for k, v in prof["phase_ms"].items()}
+    roofline = {"bound": "alu", "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "TIMAD/s",
+                "frac": achieved / peak if peak else None, "traffic": traffic,
+                "kernel": "k_accum (bucket accumulation, XYZZ madd)",
+                "algorithmic": f"{entries} bucket entries x {madd_imad(L)} IMAD (8M+2S, App. B)",
+                "peak_src": f"148 SM x 64 IMAD/clk x {sm_max:.0f} MHz ({peaks_src} sm_max)",
+                "accum_ms": accum_ms, "phase_ms_per_step": phase_share}
+    launches = int(prof["launches"]) + (1 if world > 1 else 0)
+
+    # ---- e2e: host buffers through the public API, copies inside the region ----
+    e2e = None
+    if not args.no_e2e:
+        h2d = input_bytes
+        d2h = 2 * L * 4
+        Ph = P.cpu().pin_memory()
+        Kh = K.cpu().pin_memory()
+        k_e2e = max(1, min(args.steps, 5))
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        if world == 1:
+            pn, kn = Ph.numpy().view(np.uint32), Kh.numpy().view(np.uint32)
+            outh = np.zeros(2 * L, dtype=np.uint32)
+            gz.msm_host(curve, pn, kn, outh)           # warm
+            t0 = time.perf_counter()
+            for _ in range(k_e2e):
+                gz.msm_host(curve, pn, kn, outh)       # H2D + MSM + D2H, synchronised
+            e2e_ms = (time.perf_counter() - t0) * 1e3 / k_e2e
+        else:
+            Pd = torch.empty_like(P)
+            Kd = torch.empty_like(K)
+            outh = torch.empty(2 * L, dtype=torch.int32).pin_memory()
+            t0 = time.perf_counter()
+            for _ in range(k_e2e):
+                Pd.copy_(Ph, non_blocking=True)
+                Kd.copy_(Kh, non_blocking=True)
+                o = gz.msm_sharded(curve, Pd, Kd, comm)
+                outh.copy_(o, non_blocking=True)
+                torch.cuda.synchronize()
+            e2e_ms = (time.perf_counter() - t0) * 1e3 / k_e2e
+            te = torch.tensor([e2e_ms], dtype=torch.float64, device="cuda")
+            dist.all_reduce(te, op=dist.ReduceOp.MAX)
+            e2e_ms = float(te.item())
+        e2e = {"value": n / (e2e_ms / 1e3), "unit": "points/s", "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world,
+               "api": "gzkp_msm_host" if world == 1 else "H2D + gzkp_msm_sharded + D2H"}
+
+    # ---- cpu baseline: the oracle on a bounded sample (rank 0, N = 1 only) ----
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        import oracle
+        n_s = min(n, calibrate_oracle_n(curve, 12.0))
+        rate, wall, cores, spts, sk, sout = oracle_time_sample(curve, n_s, cfg, sdist, 12.0)
+        gout = gz.to_numpy(gz.msm(curve, gz.to_device(spts), gz.to_device(sk)))
+        cpu = {"value": rate, "unit": "points/s", "cores": cores, "kind": "oracle",
+               "sample": f"{n_s} points of {wl} (scalars = the workload's first {n_s}; points tiled "
+                         f"from {min(n_s, max(8, 16 * cores))} oracle a_i*G), wall {wall:.1f} s",
+               "sample_parity_gpu_vs_oracle": bool(np.array_equal(gout, sout))}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "points/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "u32 (exact F_p, Montgomery)",
+            "data": "synthetic (seeded scalars; points a_i*G generated on device)",
+            "config": {"workload": wl, "curve": curve, "n": n, "scalars": sdist, "baseline_config": desc,
+                       "window_bits": int(prof["c"]), "parallelism": f"shard{world}" if world > 1 else "single",
+                       "l2": "flushed between steps" if flush_l2 else f"inputs {input_bytes >> 20} MiB/GPU > L2"},
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+            "gpu_launches": launches * args.steps,
+        }
+        print(json.dumps(line), flush=True)
+    if comm is not None:
+        comm.destroy()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

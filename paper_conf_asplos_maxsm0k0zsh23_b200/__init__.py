@@ -1,0 +1,362 @@
+"""B200-native G1 multi-scalar multiplication (GZKP, ASPLOS '23 -> sm_100a).
+
+Thin ctypes binding over libgzkp.so (include/gzkp.h).  Argument marshalling
+only: every step of the MSM runs in the library's CUDA kernels.  PyTorch is
+used for device memory, streams and process groups.  There is no CPU fallback:
+if libgzkp.so is missing or no CUDA device is present the calls raise.
+"""
+
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libgzkp.so")
+
+CURVES = {"bn254": 0, "bls12_381": 1, "mnt4_753": 2, "toy_a0": 100, "toy_a2": 101}
+NAMES = {v: k for k, v in CURVES.items()}
+
+_lib = None
+
+
+class GzkpError(RuntimeError):
+    pass
+
+
+def curve_id(curve) -> int:
+    if isinstance(curve, int):
+        if curve not in NAMES:
+            raise ValueError(f"unknown curve id {curve}")
+        return curve
+    name = getattr(curve, "name", curve)
+    return CURVES[name]
+
+
+def lib():
+    """Load libgzkp.so (raises if it was not built -- no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise GzkpError(f"{LIB_PATH} not built; run python -m paper_conf_asplos_maxsm0k0zsh23_b200.build")
+        L = ctypes.CDLL(LIB_PATH)
+        vp, sz, i32 = ctypes.c_void_p, ctypes.c_size_t, ctypes.c_int
+        sigs = {
+            "gzkp_field_bytes": ([i32], sz),
+            "gzkp_scalar_bytes": ([i32], sz),
+            "gzkp_partial_bytes": ([i32], sz),
+            "gzkp_msm": ([i32, vp, vp, sz, vp, vp], i32),
+            "gzkp_msm_workspace_bytes": ([i32, sz], sz),
+            "gzkp_msm_ex": ([i32, vp, vp, sz, vp, vp, sz, vp], i32),
+            "gzkp_msm_host": ([i32, vp, vp, sz, vp, vp], i32),
+            "gzkp_points_prepare": ([i32, vp, sz, ctypes.POINTER(vp), vp], i32),
+            "gzkp_msm_prepared": ([vp, vp, sz, vp, vp], i32),
+            "gzkp_msm_prepared_host": ([vp, vp, sz, vp, vp], i32),
+            "gzkp_points_release": ([vp], i32),
+            "gzkp_msm_partial": ([i32, vp, vp, sz, vp, vp], i32),
+            "gzkp_combine_partials": ([i32, vp, i32, vp, vp], i32),
+            "gzkp_nccl_unique_id": ([ctypes.c_char_p], i32),
+            "gzkp_comm_init": ([i32, i32, ctypes.c_char_p, ctypes.POINTER(vp)], i32),
+            "gzkp_comm_destroy": ([vp], i32),
+            "gzkp_msm_sharded": ([i32, vp, vp, sz, vp, vp, vp], i32),
+            "gzkp_fixed_base_mul": ([i32, vp, sz, vp, vp], i32),
+            "gzkp_field_op": ([i32, i32, vp, vp, vp, sz, vp], i32),
+            "gzkp_ec_op": ([i32, i32, vp, vp, vp, sz, vp], i32),
+            "gzkp_set_config": ([i32, i32], i32),
+            "gzkp_window_bits": ([i32, sz], i32),
+            "gzkp_set_profiling": ([i32], i32),
+            "gzkp_profile_read": ([ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_uint64), i32], i32),
+            "gzkp_status_string": ([i32], ctypes.c_char_p),
+            "gzkp_last_error": ([], ctypes.c_char_p),
+        }
+        for name, (args, res) in sigs.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = res
+        _lib = L
+    return _lib
+
+
+def _check(status: int, what: str):
+    if status:
+        L = lib()
+        raise GzkpError(f"{what}: {L.gzkp_status_string(status).decode()} "
+                        f"({L.gzkp_last_error().decode()})")
+
+
+def field_limbs(curve) -> int:
+    return lib().gzkp_field_bytes(curve_id(curve)) // 4
+
+
+def scalar_limbs(curve) -> int:
+    return lib().gzkp_scalar_bytes(curve_id(curve)) // 4
+
+
+def window_bits(curve, n: int) -> int:
+    return lib().gzkp_window_bits(curve_id(curve), n)
+
+
+def workspace_bytes(curve, n: int) -> int:
+    return lib().gzkp_msm_workspace_bytes(curve_id(curve), n)
+
+
+def set_config(window_bits: int = 0, chunk_entries: int = 0):
+    _check(lib().gzkp_set_config(window_bits, chunk_entries), "gzkp_set_config")
+
+
+PHASES = ["sort", "accumulate", "merge", "reduce", "tail"]
+
+
+def set_profiling(on: bool):
+    _check(lib().gzkp_set_profiling(1 if on else 0), "gzkp_set_profiling")
+
+
+def profile_read(reset: bool = True):
+    """Summed per-phase device ms since the last reset (CUDA events recorded on
+    the call's stream) and stats of the last call."""
+    ms = (ctypes.c_double * 5)()
+    st = (ctypes.c_uint64 * 4)()
+    _check(lib().gzkp_profile_read(ms, st, 1 if reset else 0), "gzkp_profile_read")
+    return {"phase_ms": dict(zip(PHASES, list(ms))), "calls": st[0], "launches": st[1],
+            "entries": st[2], "c": st[3]}
+
+
+# ------------------------------------------------------------ torch plumbing
+
+def _torch():
+    import torch
+    return torch
+
+
+def _stream_ptr(stream=None) -> int:
+    torch = _torch()
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return s.cuda_stream
+
+
+def _dev_u32(x, cols: int, name: str):
+    """Return a contiguous int32 CUDA tensor viewed as [n, cols] u32 limbs."""
+    torch = _torch()
+    if isinstance(x, np.ndarray):
+        x = torch.from_numpy(np.ascontiguousarray(x, dtype=np.uint32).view(np.int32))
+    if not x.is_cuda:
+        raise GzkpError(f"{name} must be a CUDA tensor (no CPU path)")
+    if x.dtype in (torch.uint8,):
+        x = x.view(torch.int32)
+    if x.dtype not in (torch.int32, torch.uint32):
+        raise GzkpError(f"{name}: expected int32/uint32/uint8 limbs, got {x.dtype}")
+    x = x.contiguous().reshape(-1, cols)
+    if x.data_ptr() % 16:
+        raise GzkpError(f"{name} must be 16-byte aligned")
+    return x
+
+
+def to_device(a: np.ndarray, device="cuda"):
+    torch = _torch()
+    return torch.from_numpy(np.ascontiguousarray(a, dtype=np.uint32).view(np.int32)).to(device)
+
+
+def to_numpy(t) -> np.ndarray:
+    return t.detach().cpu().numpy().view(np.uint32)
+
+
+def msm(curve, points, scalars, out=None, stream=None, workspace=None):
+    """Q = sum_i scalars[i] * points[i] on the current CUDA device.
+
+    points: [n, 2L] u32 limbs (canonical affine, (0,0) = O); scalars: [n, Ls].
+    Returns a [2L] int32 CUDA tensor (canonical affine, little-endian limbs)."""
+    torch = _torch()
+    cid = curve_id(curve)
+    L, Ls = field_limbs(cid), scalar_limbs(cid)
+    P = _dev_u32(points, 2 * L, "points")
+    K = _dev_u32(scalars, Ls, "scalars")
+    n = P.shape[0]
+    if K.shape[0] != n:
+        raise GzkpError("points and scalars differ in length")
+    if out is None:
+        out = torch.empty(2 * L, dtype=torch.int32, device=P.device)
+    if workspace is None:
+        st = lib().gzkp_msm(cid, P.data_ptr(), K.data_ptr(), n, out.data_ptr(), _stream_ptr(stream))
+    else:
+        st = lib().gzkp_msm_ex(cid, P.data_ptr(), K.data_ptr(), n, out.data_ptr(), workspace.data_ptr(),
+                               workspace.numel() * workspace.element_size(), _stream_ptr(stream))
+    _check(st, "gzkp_msm")
+    return out
+
+
+def msm_host(curve, points: np.ndarray, scalars: np.ndarray, out: Optional[np.ndarray] = None, stream=None):
+    """MSM from HOST buffers: copies inside the call (the e2e path)."""
+    cid = curve_id(curve)
+    L = field_limbs(cid)
+    points = np.ascontiguousarray(points, dtype=np.uint32)
+    scalars = np.ascontiguousarray(scalars, dtype=np.uint32)
+    n = points.shape[0] if points.ndim == 2 else points.size // (2 * L)
+    if out is None:
+        out = np.zeros(2 * L, dtype=np.uint32)
+    st = lib().gzkp_msm_host(cid, points.ctypes.data, scalars.ctypes.data, n, out.ctypes.data, _stream_ptr(stream))
+    _check(st, "gzkp_msm_host")
+    return out
+
+
+class PreparedPoints:
+    """Device-resident Montgomery copy of a fixed point vector."""
+
+    def __init__(self, curve, points, stream=None):
+        self.curve = curve_id(curve)
+        L = field_limbs(self.curve)
+        P = _dev_u32(points, 2 * L, "points")
+        self.n = P.shape[0]
+        h = ctypes.c_void_p()
+        _check(lib().gzkp_points_prepare(self.curve, P.data_ptr(), self.n, ctypes.byref(h), _stream_ptr(stream)),
+               "gzkp_points_prepare")
+        self.handle = h
+
+    def msm(self, scalars, out=None, stream=None):
+        torch = _torch()
+        L, Ls = field_limbs(self.curve), scalar_limbs(self.curve)
+        K = _dev_u32(scalars, Ls, "scalars")
+        if out is None:
+            out = torch.empty(2 * L, dtype=torch.int32, device=K.device)
+        _check(lib().gzkp_msm_prepared(self.handle, K.data_ptr(), K.shape[0], out.data_ptr(), _stream_ptr(stream)),
+               "gzkp_msm_prepared")
+        return out
+
+    def msm_host(self, scalars: np.ndarray, out: Optional[np.ndarray] = None, stream=None):
+        L = field_limbs(self.curve)
+        scalars = np.ascontiguousarray(scalars, dtype=np.uint32)
+        if out is None:
+            out = np.zeros(2 * L, dtype=np.uint32)
+        _check(lib().gzkp_msm_prepared_host(self.handle, scalars.ctypes.data, scalars.shape[0], out.ctypes.data,
+                                            _stream_ptr(stream)), "gzkp_msm_prepared_host")
+        return out
+
+    def release(self):
+        if self.handle:
+            lib().gzkp_points_release(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.release()
+        except Exception:
+            pass
+
+
+def msm_partial(curve, points, scalars, out=None, stream=None):
+    torch = _torch()
+    cid = curve_id(curve)
+    L, Ls = field_limbs(cid), scalar_limbs(cid)
+    P = _dev_u32(points, 2 * L, "points")
+    K = _dev_u32(scalars, Ls, "scalars")
+    if out is None:
+        out = torch.empty(4 * L, dtype=torch.int32, device=P.device)
+    _check(lib().gzkp_msm_partial(cid, P.data_ptr(), K.data_ptr(), P.shape[0], out.data_ptr(), _stream_ptr(stream)),
+           "gzkp_msm_partial")
+    return out
+
+
+def combine_partials(curve, partials, out=None, stream=None):
+    torch = _torch()
+    cid = curve_id(curve)
+    L = field_limbs(cid)
+    Pt = _dev_u32(partials, 4 * L, "partials")
+    if out is None:
+        out = torch.empty(2 * L, dtype=torch.int32, device=Pt.device)
+    _check(lib().gzkp_combine_partials(cid, Pt.data_ptr(), Pt.shape[0], out.data_ptr(), _stream_ptr(stream)),
+           "gzkp_combine_partials")
+    return out
+
+
+def fixed_base_mul(curve, scalars, out=None, stream=None):
+    """out[i] = scalars[i] * G (canonical affine) -- synthetic key generation."""
+    torch = _torch()
+    cid = curve_id(curve)
+    L, Ls = field_limbs(cid), scalar_limbs(cid)
+    K = _dev_u32(scalars, Ls, "scalars")
+    if out is None:
+        out = torch.empty((K.shape[0], 2 * L), dtype=torch.int32, device=K.device)
+    _check(lib().gzkp_fixed_base_mul(cid, K.data_ptr(), K.shape[0], out.data_ptr(), _stream_ptr(stream)),
+           "gzkp_fixed_base_mul")
+    return out
+
+
+def field_op(curve, op: int, a, b, stream=None):
+    torch = _torch()
+    cid = curve_id(curve)
+    L = field_limbs(cid)
+    A = _dev_u32(a, L, "a")
+    B = _dev_u32(b, L, "b")
+    out = torch.empty_like(A)
+    _check(lib().gzkp_field_op(cid, op, A.data_ptr(), B.data_ptr(), out.data_ptr(), A.shape[0], _stream_ptr(stream)),
+           "gzkp_field_op")
+    return out
+
+
+def ec_op(curve, op: int, P, Q, stream=None):
+    torch = _torch()
+    cid = curve_id(curve)
+    L = field_limbs(cid)
+    A = _dev_u32(P, 2 * L, "P")
+    B = _dev_u32(Q, 2 * L, "Q")
+    out = torch.empty_like(A)
+    _check(lib().gzkp_ec_op(cid, op, A.data_ptr(), B.data_ptr(), out.data_ptr(), A.shape[0], _stream_ptr(stream)),
+           "gzkp_ec_op")
+    return out
+
+
+# ------------------------------------------------------------- multi-GPU
+
+class Comm:
+    """NCCL communicator for gzkp_msm_sharded.  The 128-byte unique id is
+    broadcast through the default torch process group (plumbing only)."""
+
+    def __init__(self, world: int, rank: int, group=None):
+        torch = _torch()
+        import torch.distributed as dist
+        uid = ctypes.create_string_buffer(128)
+        if rank == 0:
+            _check(lib().gzkp_nccl_unique_id(uid), "gzkp_nccl_unique_id")
+        t = torch.frombuffer(bytearray(uid.raw), dtype=torch.uint8).clone()
+        if dist.get_backend(group) == "nccl":
+            t = t.cuda()
+        dist.broadcast(t, src=0, group=group)
+        raw = bytes(t.cpu().numpy().tobytes())
+        uid = ctypes.create_string_buffer(raw, 128)
+        h = ctypes.c_void_p()
+        _check(lib().gzkp_comm_init(world, rank, uid, ctypes.byref(h)), "gzkp_comm_init")
+        self.handle = h
+        self.world, self.rank = world, rank
+
+    def destroy(self):
+        if self.handle:
+            lib().gzkp_comm_destroy(self.handle)
+            self.handle = None
+
+
+def shard_range(n: int, world: int, rank: int):
+    """Contiguous slice [lo, hi) of rank `rank`."""
+    per = (n + world - 1) // world if world else 0
+    lo = min(n, rank * per)
+    hi = min(n, (rank + 1) * per)
+    return lo, hi
+
+
+def msm_sharded(curve, points_local, scalars_local, comm: Comm, out=None, stream=None):
+    torch = _torch()
+    cid = curve_id(curve)
+    L, Ls = field_limbs(cid), scalar_limbs(cid)
+    P = _dev_u32(points_local, 2 * L, "points")
+    K = _dev_u32(scalars_local, Ls, "scalars")
+    if out is None:
+        out = torch.empty(2 * L, dtype=torch.int32, device=P.device)
+    _check(lib().gzkp_msm_sharded(cid, P.data_ptr(), K.data_ptr(), P.shape[0], out.data_ptr(), _stream_ptr(stream),
+                                  comm.handle), "gzkp_msm_sharded")
+    return out
+
+
+__all__ = ["CURVES", "GzkpError", "lib", "msm", "msm_host", "PreparedPoints", "msm_partial", "combine_partials",
+           "fixed_base_mul", "field_op", "ec_op", "Comm", "msm_sharded", "shard_range", "set_config",
+           "window_bits", "workspace_bytes", "set_profiling", "profile_read", "field_limbs", "scalar_limbs", "to_device", "to_numpy"]

@@ -1,0 +1,480 @@
+// abi.cu -- the extern "C" boundary of libgzkp.so (declared in include/gzkp.h).
+//
+// Argument checking, curve dispatch, prepared-point handles, host-buffer
+// wrappers, and the multi-GPU path (one NCCL all-gather of per-rank XYZZ
+// partials, §5.2).  No exception crosses this boundary.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "internal.h"
+
+namespace gzkp {
+
+static thread_local std::string g_last_error;
+
+Tunables& tunables() {
+  static Tunables t;
+  return t;
+}
+
+gzkp_status set_error(gzkp_status st, const std::string& msg) {
+  g_last_error = msg;
+  return st;
+}
+
+gzkp_status cuda_status(cudaError_t e, const char* where) {
+  g_last_error = std::string(where) + ": " + cudaGetErrorString(e);
+  return e == cudaErrorMemoryAllocation ? GZKP_ERROR_OUT_OF_MEMORY : GZKP_ERROR_CUDA;
+}
+
+int device_sm_count() {
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  return sms > 0 ? sms : 148;
+}
+
+static int g_profiling = -1;
+bool profiling_enabled() {
+  if (g_profiling < 0) {
+    const char* e = getenv("GZKP_PROFILE");
+    g_profiling = (e && atoi(e) != 0) ? 1 : 0;
+  }
+  return g_profiling == 1;
+}
+
+// pending records of this thread, harvested by gzkp_profile_read
+static thread_local std::vector<ProfileRecord*> g_pending;
+static thread_local double g_phase_sum[5] = {0, 0, 0, 0, 0};
+static thread_local uint64_t g_calls = 0, g_last_launches = 0, g_last_entries = 0, g_last_c = 0;
+
+ProfileRecord* profile_begin(cudaStream_t s) {
+  if (!profiling_enabled()) return nullptr;
+  // one pinned word per thread, allocated on first use (every record writes
+  // the entry count of its call there; only the last call's value is read)
+  static thread_local uint32_t* pinned = nullptr;
+  if (!pinned && cudaMallocHost((void**)&pinned, sizeof(uint32_t)) != cudaSuccess) return nullptr;
+  ProfileRecord* r = new ProfileRecord;
+  for (auto& e : r->ev) cudaEventCreate(&e);
+  r->entries_host = pinned;
+  r->launches = 0;
+  r->c = 0;
+  cudaEventRecord(r->ev[0], s);
+  return r;
+}
+void profile_mark(ProfileRecord* r, int i, cudaStream_t s) {
+  if (r) cudaEventRecord(r->ev[i], s);
+}
+void profile_end(ProfileRecord* r, const uint32_t* entries_dev, int launches, int c, cudaStream_t s) {
+  if (!r) return;
+  cudaEventRecord(r->ev[5], s);
+  cudaMemcpyAsync(r->entries_host, entries_dev, sizeof(uint32_t), cudaMemcpyDeviceToHost, s);
+  r->launches = launches;
+  r->c = c;
+  g_pending.push_back(r);
+}
+
+const CurveImpl* impl_for(int curve) {
+  switch (curve) {
+    case GZKP_BN254: return impl_bn254();
+    case GZKP_BLS12_381: return impl_bls12_381();
+    case GZKP_MNT4_753: return impl_mnt4_753();
+    case GZKP_TOY_A0: return impl_toy_a0();
+    case GZKP_TOY_A2: return impl_toy_a2();
+    default: return nullptr;
+  }
+}
+
+// the stream-ordered pool keeps freed workspace (no re-allocation per call)
+static void init_pool_once() {
+  static std::once_flag once;
+  std::call_once(once, [] {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+      uint64_t thr = UINT64_MAX;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  });
+}
+
+static bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
+
+struct Prepared {
+  int curve;
+  size_t n;
+  void* pts;   // Montgomery affine, n x 2N u32
+};
+
+// ------------------------------------------------------------- NCCL (dlopen)
+// NCCL is resolved at run time so libgzkp.so loads without it; when torch has
+// already loaded its libnccl.so.2 the same copy is reused (RTLD_NOLOAD first).
+typedef struct ncclComm* ncclComm_t;
+typedef struct { char internal[128]; } ncclUniqueId;
+typedef int ncclResult_t;
+enum { ncclUint8_ = 1 };
+
+struct Nccl {
+  void* h = nullptr;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*AllGather)(const void*, void*, size_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+  bool ok = false;
+};
+
+static Nccl& nccl() {
+  static Nccl n;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    const char* names[] = {"libnccl.so.2", "libnccl.so"};
+    for (const char* nm : names) {
+      n.h = dlopen(nm, RTLD_NOW | RTLD_NOLOAD);
+      if (n.h) break;
+    }
+    if (!n.h) {
+      for (const char* nm : names) {
+        n.h = dlopen(nm, RTLD_NOW | RTLD_GLOBAL);
+        if (n.h) break;
+      }
+    }
+    if (!n.h) return;
+    n.GetUniqueId = (decltype(n.GetUniqueId))dlsym(n.h, "ncclGetUniqueId");
+    n.CommInitRank = (decltype(n.CommInitRank))dlsym(n.h, "ncclCommInitRank");
+    n.CommDestroy = (decltype(n.CommDestroy))dlsym(n.h, "ncclCommDestroy");
+    n.AllGather = (decltype(n.AllGather))dlsym(n.h, "ncclAllGather");
+    n.GetErrorString = (decltype(n.GetErrorString))dlsym(n.h, "ncclGetErrorString");
+    n.ok = n.GetUniqueId && n.CommInitRank && n.CommDestroy && n.AllGather;
+  });
+  return n;
+}
+
+struct Comm {
+  ncclComm_t comm = nullptr;
+  int world = 1, rank = 0;
+  void* partial = nullptr;    // 4N u32 (max N)
+  void* gathered = nullptr;   // world x 4N u32
+};
+
+static gzkp_status nccl_status(ncclResult_t r, const char* where) {
+  if (r == 0) return GZKP_SUCCESS;
+  std::string m = std::string(where) + ": nccl error " + std::to_string(r);
+  if (nccl().GetErrorString) m += std::string(" (") + nccl().GetErrorString(r) + ")";
+  return set_error(GZKP_ERROR_NCCL, m);
+}
+
+}  // namespace gzkp
+
+using namespace gzkp;
+
+extern "C" {
+
+size_t gzkp_field_bytes(int curve) {
+  const CurveImpl* c = impl_for(curve);
+  return c ? (size_t)c->limbs * 4 : 0;
+}
+size_t gzkp_scalar_bytes(int curve) {
+  const CurveImpl* c = impl_for(curve);
+  return c ? (size_t)c->scalar_limbs * 4 : 0;
+}
+size_t gzkp_partial_bytes(int curve) {
+  const CurveImpl* c = impl_for(curve);
+  return c ? (size_t)c->limbs * 16 : 0;
+}
+
+int gzkp_window_bits(int curve, size_t n) {
+  const CurveImpl* c = impl_for(curve);
+  return c ? c->window_bits(n) : -1;
+}
+
+size_t gzkp_msm_workspace_bytes(int curve, size_t n) {
+  const CurveImpl* c = impl_for(curve);
+  return c ? c->workspace_bytes(n, false) : 0;
+}
+
+static gzkp_status check_args(const CurveImpl* c, const void* pts, const void* sc, size_t n, const void* out) {
+  if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
+  if (!out) return set_error(GZKP_ERROR_INVALID_VALUE, "out is NULL");
+  if (n && (!pts || !sc)) return set_error(GZKP_ERROR_INVALID_VALUE, "NULL input with n > 0");
+  if (!aligned16(pts) || !aligned16(sc) || !aligned16(out))
+    return set_error(GZKP_ERROR_INVALID_VALUE, "buffers must be 16-byte aligned");
+  return GZKP_SUCCESS;
+}
+
+gzkp_status gzkp_msm_ex(int curve, const void* points_affine, const void* scalars, size_t n, void* out,
+                        void* workspace, size_t workspace_bytes, gzkp_stream stream) {
+  const CurveImpl* c = impl_for(curve);
+  if (gzkp_status st = check_args(c, points_affine, scalars, n, out)) return st;
+  init_pool_once();
+  MsmCall call;
+  call.points = points_affine;
+  call.scalars = scalars;
+  call.n = n;
+  call.out_affine = out;
+  call.workspace = workspace;
+  call.workspace_bytes = workspace_bytes;
+  call.stream = (cudaStream_t)stream;
+  return c->msm(call);
+}
+
+gzkp_status gzkp_msm(int curve, const void* points_affine, const void* scalars, size_t n, void* out,
+                     gzkp_stream stream) {
+  return gzkp_msm_ex(curve, points_affine, scalars, n, out, nullptr, 0, stream);
+}
+
+gzkp_status gzkp_msm_partial(int curve, const void* points_affine, const void* scalars, size_t n,
+                             void* partial_xyzz, gzkp_stream stream) {
+  const CurveImpl* c = impl_for(curve);
+  if (gzkp_status st = check_args(c, points_affine, scalars, n, partial_xyzz)) return st;
+  init_pool_once();
+  MsmCall call;
+  call.points = points_affine;
+  call.scalars = scalars;
+  call.n = n;
+  call.out_partial = partial_xyzz;
+  call.stream = (cudaStream_t)stream;
+  return c->msm(call);
+}
+
+gzkp_status gzkp_combine_partials(int curve, const void* partials_xyzz, int count, void* out_affine,
+                                  gzkp_stream stream) {
+  const CurveImpl* c = impl_for(curve);
+  if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
+  if (count < 0 || !out_affine || (count && !partials_xyzz)) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
+  return c->combine(partials_xyzz, count, out_affine, (cudaStream_t)stream);
+}
+
+gzkp_status gzkp_msm_host(int curve, const void* points_host, const void* scalars_host, size_t n, void* out_host,
+                          gzkp_stream stream) {
+  const CurveImpl* c = impl_for(curve);
+  if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
+  if (!out_host || (n && (!points_host || !scalars_host))) return set_error(GZKP_ERROR_INVALID_VALUE, "NULL argument");
+  init_pool_once();
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t pb = n * 2 * c->limbs * 4, sb = n * c->scalar_limbs * 4, ob = 2 * c->limbs * 4;
+  char* d = nullptr;
+  const size_t total = align_up(pb) + align_up(sb) + align_up(ob);
+  cudaError_t e = cudaMallocAsync((void**)&d, total, s);
+  if (e != cudaSuccess) return cuda_status(e, "cudaMallocAsync");
+  void *dp = d, *ds = d + align_up(pb), *dout = d + align_up(pb) + align_up(sb);
+  gzkp_status st = GZKP_SUCCESS;
+  if (n && (e = cudaMemcpyAsync(dp, points_host, pb, cudaMemcpyHostToDevice, s)) != cudaSuccess) st = cuda_status(e, "H2D points");
+  if (!st && n && (e = cudaMemcpyAsync(ds, scalars_host, sb, cudaMemcpyHostToDevice, s)) != cudaSuccess) st = cuda_status(e, "H2D scalars");
+  if (!st) st = gzkp_msm(curve, dp, ds, n, dout, stream);
+  if (!st && (e = cudaMemcpyAsync(out_host, dout, ob, cudaMemcpyDeviceToHost, s)) != cudaSuccess) st = cuda_status(e, "D2H out");
+  cudaFreeAsync(d, s);
+  if ((e = cudaStreamSynchronize(s)) != cudaSuccess && !st) st = cuda_status(e, "cudaStreamSynchronize");
+  return st;
+}
+
+gzkp_status gzkp_points_prepare(int curve, const void* points_affine, size_t n, void** handle, gzkp_stream stream) {
+  const CurveImpl* c = impl_for(curve);
+  if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
+  if (!handle || (n && !points_affine) || !aligned16(points_affine))
+    return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
+  Prepared* h = new (std::nothrow) Prepared{curve, n, nullptr};
+  if (!h) return set_error(GZKP_ERROR_OUT_OF_MEMORY, "handle");
+  if (n) {
+    cudaError_t e = cudaMalloc(&h->pts, n * 2 * c->limbs * 4);
+    if (e != cudaSuccess) { delete h; return cuda_status(e, "cudaMalloc(prepared)"); }
+    gzkp_status st = c->to_mont(points_affine, h->pts, n, (cudaStream_t)stream);
+    if (st) { cudaFree(h->pts); delete h; return st; }
+  }
+  *handle = h;
+  return GZKP_SUCCESS;
+}
+
+gzkp_status gzkp_msm_prepared(const void* handle, const void* scalars, size_t n, void* out, gzkp_stream stream) {
+  const Prepared* h = (const Prepared*)handle;
+  if (!h) return set_error(GZKP_ERROR_INVALID_VALUE, "NULL handle");
+  if (n > h->n) return set_error(GZKP_ERROR_INVALID_VALUE, "n exceeds prepared point count");
+  const CurveImpl* c = impl_for(h->curve);
+  if (gzkp_status st = check_args(c, h->pts, scalars, n, out)) return st;
+  init_pool_once();
+  MsmCall call;
+  call.points = h->pts;
+  call.prepared = true;
+  call.scalars = scalars;
+  call.n = n;
+  call.out_affine = out;
+  call.stream = (cudaStream_t)stream;
+  return c->msm(call);
+}
+
+gzkp_status gzkp_msm_prepared_host(const void* handle, const void* scalars_host, size_t n, void* out_host,
+                                   gzkp_stream stream) {
+  const Prepared* h = (const Prepared*)handle;
+  if (!h) return set_error(GZKP_ERROR_INVALID_VALUE, "NULL handle");
+  const CurveImpl* c = impl_for(h->curve);
+  if (!c || !out_host || (n && !scalars_host)) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t sb = n * c->scalar_limbs * 4, ob = 2 * c->limbs * 4;
+  char* d = nullptr;
+  cudaError_t e = cudaMallocAsync((void**)&d, align_up(sb) + align_up(ob), s);
+  if (e != cudaSuccess) return cuda_status(e, "cudaMallocAsync");
+  void *ds = d, *dout = d + align_up(sb);
+  gzkp_status st = GZKP_SUCCESS;
+  if (n && (e = cudaMemcpyAsync(ds, scalars_host, sb, cudaMemcpyHostToDevice, s)) != cudaSuccess) st = cuda_status(e, "H2D scalars");
+  if (!st) st = gzkp_msm_prepared(handle, ds, n, dout, stream);
+  if (!st && (e = cudaMemcpyAsync(out_host, dout, ob, cudaMemcpyDeviceToHost, s)) != cudaSuccess) st = cuda_status(e, "D2H out");
+  cudaFreeAsync(d, s);
+  if ((e = cudaStreamSynchronize(s)) != cudaSuccess && !st) st = cuda_status(e, "cudaStreamSynchronize");
+  return st;
+}
+
+gzkp_status gzkp_points_release(void* handle) {
+  Prepared* h = (Prepared*)handle;
+  if (!h) return GZKP_SUCCESS;
+  if (h->pts) cudaFree(h->pts);
+  delete h;
+  return GZKP_SUCCESS;
+}
+
+gzkp_status gzkp_fixed_base_mul(int curve, const void* scalars, size_t n, void* out_affine, gzkp_stream stream) {
+  const CurveImpl* c = impl_for(curve);
+  if (gzkp_status st = check_args(c, out_affine, scalars, n, out_affine)) return st;
+  return c->fixed_base(scalars, n, out_affine, (cudaStream_t)stream);
+}
+
+gzkp_status gzkp_field_op(int curve, int op, const void* a, const void* b, void* out, size_t n, gzkp_stream stream) {
+  const CurveImpl* c = impl_for(curve);
+  if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
+  if (op < 0 || op > 4 || (n && (!a || !b || !out))) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
+  return c->field_op(op, a, b, out, n, (cudaStream_t)stream);
+}
+
+gzkp_status gzkp_ec_op(int curve, int op, const void* P, const void* Q, void* out, size_t n, gzkp_stream stream) {
+  const CurveImpl* c = impl_for(curve);
+  if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
+  if (op < 0 || op > 3 || (n && (!P || !Q || !out))) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
+  return c->ec_op(op, P, Q, out, n, (cudaStream_t)stream);
+}
+
+gzkp_status gzkp_set_config(int window_bits, int chunk_entries) {
+  if (window_bits < 0 || window_bits > 16 || window_bits == 1 || chunk_entries < 0 || chunk_entries > (1 << 20))
+    return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..16");
+  tunables().window_bits = window_bits;
+  tunables().chunk_entries = chunk_entries;
+  return GZKP_SUCCESS;
+}
+
+gzkp_status gzkp_set_profiling(int on) {
+  g_profiling = on ? 1 : 0;
+  return GZKP_SUCCESS;
+}
+
+gzkp_status gzkp_profile_read(double phase_ms[5], uint64_t stats[4], int reset) {
+  for (ProfileRecord* r : g_pending) {
+    cudaEventSynchronize(r->ev[5]);
+    for (int i = 0; i < 5; ++i) {
+      float ms = 0.f;
+      cudaEventElapsedTime(&ms, r->ev[i], r->ev[i + 1]);
+      g_phase_sum[i] += ms;
+    }
+    ++g_calls;
+    g_last_launches = r->launches;
+    g_last_entries = *r->entries_host;
+    g_last_c = r->c;
+    for (auto& e : r->ev) cudaEventDestroy(e);
+    delete r;
+  }
+  g_pending.clear();
+  if (phase_ms)
+    for (int i = 0; i < 5; ++i) phase_ms[i] = g_phase_sum[i];
+  if (stats) {
+    stats[0] = g_calls;
+    stats[1] = g_last_launches;
+    stats[2] = g_last_entries;
+    stats[3] = g_last_c;
+  }
+  if (reset) {
+    for (int i = 0; i < 5; ++i) g_phase_sum[i] = 0;
+    g_calls = 0;
+  }
+  return GZKP_SUCCESS;
+}
+
+// ------------------------------------------------------------- multi-GPU
+gzkp_status gzkp_nccl_unique_id(unsigned char id[128]) {
+  Nccl& n = nccl();
+  if (!n.ok) return set_error(GZKP_ERROR_NCCL, "libnccl.so.2 not found");
+  ncclUniqueId u;
+  if (gzkp_status st = nccl_status(n.GetUniqueId(&u), "ncclGetUniqueId")) return st;
+  memcpy(id, u.internal, 128);
+  return GZKP_SUCCESS;
+}
+
+gzkp_status gzkp_comm_init(int world, int rank, const unsigned char id[128], void** comm) {
+  Nccl& n = nccl();
+  if (!n.ok) return set_error(GZKP_ERROR_NCCL, "libnccl.so.2 not found");
+  if (world < 1 || rank < 0 || rank >= world || !id || !comm) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
+  Comm* c = new (std::nothrow) Comm;
+  if (!c) return set_error(GZKP_ERROR_OUT_OF_MEMORY, "comm");
+  c->world = world;
+  c->rank = rank;
+  ncclUniqueId u;
+  memcpy(u.internal, id, 128);
+  if (gzkp_status st = nccl_status(n.CommInitRank(&c->comm, world, u, rank), "ncclCommInitRank")) { delete c; return st; }
+  const size_t pmax = 24 * 16;   // largest XYZZ partial (MNT4-753)
+  cudaError_t e;
+  if ((e = cudaMalloc(&c->partial, pmax)) != cudaSuccess || (e = cudaMalloc(&c->gathered, pmax * world)) != cudaSuccess) {
+    n.CommDestroy(c->comm);
+    delete c;
+    return cuda_status(e, "cudaMalloc(comm buffers)");
+  }
+  *comm = c;
+  return GZKP_SUCCESS;
+}
+
+gzkp_status gzkp_comm_destroy(void* comm) {
+  Comm* c = (Comm*)comm;
+  if (!c) return GZKP_SUCCESS;
+  if (c->comm && nccl().ok) nccl().CommDestroy(c->comm);
+  cudaFree(c->partial);
+  cudaFree(c->gathered);
+  delete c;
+  return GZKP_SUCCESS;
+}
+
+gzkp_status gzkp_msm_sharded(int curve, const void* points_affine, const void* scalars, size_t n_local, void* out,
+                             gzkp_stream stream, void* comm) {
+  Comm* cm = (Comm*)comm;
+  const CurveImpl* c = impl_for(curve);
+  if (!cm) return set_error(GZKP_ERROR_INVALID_VALUE, "NULL comm");
+  if (gzkp_status st = check_args(c, points_affine, scalars, n_local, out)) return st;
+  cudaStream_t s = (cudaStream_t)stream;
+  // 1. full Pippenger on this rank's shard -> XYZZ partial
+  if (gzkp_status st = gzkp_msm_partial(curve, points_affine, scalars, n_local, cm->partial, stream)) return st;
+  // 2. the one collective: all-gather of the per-rank partials (rank order)
+  const size_t pb = gzkp_partial_bytes(curve);
+  if (gzkp_status st = nccl_status(nccl().AllGather(cm->partial, cm->gathered, pb, ncclUint8_, cm->comm, s), "ncclAllGather"))
+    return st;
+  // 3. fold in rank order + normalise; identical bytes on every rank
+  return c->combine(cm->gathered, cm->world, out, s);
+}
+
+const char* gzkp_status_string(gzkp_status status) {
+  switch (status) {
+    case GZKP_SUCCESS: return "success";
+    case GZKP_ERROR_INVALID_VALUE: return "invalid value";
+    case GZKP_ERROR_UNSUPPORTED_CURVE: return "unsupported curve";
+    case GZKP_ERROR_OUT_OF_MEMORY: return "out of memory";
+    case GZKP_ERROR_CUDA: return "CUDA error";
+    case GZKP_ERROR_NCCL: return "NCCL error";
+    default: return "unknown status";
+  }
+}
+
+const char* gzkp_last_error(void) { return g_last_error.c_str(); }
+
+}  // extern "C"

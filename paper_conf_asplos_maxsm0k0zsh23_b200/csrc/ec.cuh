@@ -1,0 +1,248 @@
+// ec.cuh -- G1 group law in XYZZ coordinates (x = X/ZZ, y = Y/ZZZ, ZZ^3 = ZZZ^2).
+//
+// The paper's PADD ("point-addition ... including point doubling",
+// PAPER.md:116 fn. 2, §2.1) on E: y^2 = x^3 + a x + b.  The paper
+// does not fix a coordinate system (reading R6); XYZZ is chosen because
+// the bucket hot loop is a mixed add (affine input point) and XYZZ's madd costs
+// 8M + 2S with no inversion:
+//   madd-2008-s : XYZZ + affine        8M + 2S
+//   add-2008-s  : XYZZ + XYZZ         12M + 2S
+//   dbl-2008-s-1: 2 * XYZZ (general a)  6M + 3S (+1S +1M when a != 0)
+//   mdbl-2008-s-1: 2 * affine
+// Exceptional cases are explicit: the identity O is ZZ = ZZZ = 0 (tracked by a
+// flag in the hot loop), P == Q takes the doubling path, P == -Q gives O.  Every
+// field value is canonical, so the P == Q tests are exact limb comparisons.
+#pragma once
+#include "field.cuh"
+
+namespace gzkp {
+
+template <class C>
+struct EC {
+  static constexpr int N = C::N;
+  using Fp = F<C>;
+
+  struct Xyzz {
+    uint32_t X[N], Y[N], ZZ[N], ZZZ[N];
+  };
+
+  GZ_DEV static void set_inf(Xyzz& P) {
+    Fp::set_zero(P.X); Fp::set_one(P.Y); Fp::set_zero(P.ZZ); Fp::set_zero(P.ZZZ);
+  }
+  GZ_DEV static bool is_inf(const Xyzz& P) { return Fp::is_zero(P.ZZ); }
+
+  GZ_DEV static void from_affine(Xyzz& R, const uint32_t x[N], const uint32_t y[N]) {
+    Fp::copy(R.X, x); Fp::copy(R.Y, y); Fp::set_one(R.ZZ); Fp::set_one(R.ZZZ);
+  }
+
+  // M = 3 x^2 + a zz^2   (zz == nullptr means zz = 1)
+  GZ_DEV static void tangent_m(uint32_t M[N], const uint32_t X[N], const uint32_t* ZZ) {
+    uint32_t t[N];
+    Fp::sqr(t, X);
+    Fp::add(M, t, t);
+    Fp::add(M, M, t);
+    if constexpr (!C::A_ZERO) {
+      uint32_t a[N];
+#pragma unroll
+      for (int i = 0; i < N; ++i) a[i] = C::A_MONT(i);
+      if (ZZ) {
+        uint32_t z2[N];
+        Fp::sqr(z2, ZZ);
+        Fp::mul(t, z2, a);
+        Fp::add(M, M, t);
+      } else {
+        Fp::add(M, M, a);
+      }
+    }
+  }
+
+  // R = 2 * (x, y) for an affine point (mdbl-2008-s-1); y == 0 gives O.
+  GZ_DEV static void mdbl(Xyzz& R, const uint32_t x[N], const uint32_t y[N]) {
+    uint32_t U[N], V[N], W[N], S[N], M[N], t[N];
+    Fp::dbl(U, y);
+    Fp::sqr(V, U);
+    Fp::mul(W, U, V);
+    Fp::mul(S, x, V);
+    tangent_m(M, x, nullptr);
+    Fp::sqr(t, M);
+    Fp::sub(t, t, S);
+    Fp::sub(R.X, t, S);                 // X3 = M^2 - 2S
+    Fp::sub(t, S, R.X);
+    Fp::mul(t, M, t);
+    Fp::mul(S, W, y);
+    Fp::sub(R.Y, t, S);                 // Y3 = M(S - X3) - W y
+    Fp::copy(R.ZZ, V);
+    Fp::copy(R.ZZZ, W);
+  }
+
+  // P = 2P (dbl-2008-s-1, general a).  O and 2-torsion map to O (V = 0).
+  GZ_DEV static void dbl(Xyzz& P) {
+    uint32_t U[N], V[N], W[N], S[N], M[N], t[N];
+    Fp::dbl(U, P.Y);
+    Fp::sqr(V, U);
+    Fp::mul(W, U, V);
+    Fp::mul(S, P.X, V);
+    tangent_m(M, P.X, P.ZZ);
+    Fp::sqr(t, M);
+    Fp::sub(t, t, S);
+    Fp::sub(P.X, t, S);                 // X3 = M^2 - 2S
+    Fp::sub(t, S, P.X);
+    Fp::mul(t, M, t);
+    Fp::mul(S, W, P.Y);
+    Fp::sub(P.Y, t, S);                 // Y3 = M(S - X3) - W Y1
+    Fp::mul(P.ZZ, V, P.ZZ);
+    Fp::mul(P.ZZZ, W, P.ZZZ);
+  }
+
+  // acc += (x2, y2) affine, acc not O (madd-2008-s).  Exceptional cases explicit.
+  GZ_DEV static void madd_nz(Xyzz& A, const uint32_t x2[N], const uint32_t y2[N]) {
+    uint32_t P[N], R[N], PP[N], PPP[N], t[N];
+    Fp::mul(P, x2, A.ZZ);               // U2
+    Fp::sub(P, P, A.X);                 // P = U2 - X1
+    Fp::mul(R, y2, A.ZZZ);              // S2
+    Fp::sub(R, R, A.Y);                 // R = S2 - Y1
+    if (Fp::is_zero(P)) {
+      if (Fp::is_zero(R)) mdbl(A, x2, y2);   // same point
+      else set_inf(A);                       // inverse points
+      return;
+    }
+    Fp::sqr(PP, P);
+    Fp::mul(PPP, P, PP);
+    Fp::mul(A.ZZ, A.ZZ, PP);            // ZZ3 = ZZ1 PP
+    Fp::mul(A.ZZZ, A.ZZZ, PPP);         // ZZZ3 = ZZZ1 PPP
+    Fp::mul(PP, A.X, PP);               // Q = X1 PP
+    Fp::sqr(t, R);
+    Fp::sub(t, t, PPP);
+    Fp::sub(t, t, PP);
+    Fp::sub(A.X, t, PP);                // X3 = R^2 - PPP - 2Q
+    Fp::sub(t, PP, A.X);
+    Fp::mul(t, R, t);
+    Fp::mul(PPP, A.Y, PPP);
+    Fp::sub(A.Y, t, PPP);               // Y3 = R(Q - X3) - Y1 PPP
+  }
+
+  // acc += B (add-2008-s), all cases.
+  GZ_DEV static void add(Xyzz& A, const Xyzz& B) {
+    if (is_inf(B)) return;
+    if (is_inf(A)) { A = B; return; }
+    uint32_t U1[N], S1[N], P[N], R[N], PP[N], PPP[N], t[N];
+    Fp::mul(U1, A.X, B.ZZ);
+    Fp::mul(P, B.X, A.ZZ);
+    Fp::sub(P, P, U1);                  // P = U2 - U1
+    Fp::mul(S1, A.Y, B.ZZZ);
+    Fp::mul(R, B.Y, A.ZZZ);
+    Fp::sub(R, R, S1);                  // R = S2 - S1
+    if (Fp::is_zero(P)) {
+      if (Fp::is_zero(R)) dbl(A);
+      else set_inf(A);
+      return;
+    }
+    Fp::sqr(PP, P);
+    Fp::mul(PPP, P, PP);
+    Fp::mul(A.ZZ, A.ZZ, B.ZZ);
+    Fp::mul(A.ZZ, A.ZZ, PP);            // ZZ3 = ZZ1 ZZ2 PP
+    Fp::mul(A.ZZZ, A.ZZZ, B.ZZZ);
+    Fp::mul(A.ZZZ, A.ZZZ, PPP);         // ZZZ3 = ZZZ1 ZZZ2 PPP
+    Fp::mul(PP, U1, PP);                // Q = U1 PP
+    Fp::sqr(t, R);
+    Fp::sub(t, t, PPP);
+    Fp::sub(t, t, PP);
+    Fp::sub(A.X, t, PP);                // X3 = R^2 - PPP - 2Q
+    Fp::sub(t, PP, A.X);
+    Fp::mul(t, R, t);
+    Fp::mul(PPP, S1, PPP);
+    Fp::sub(A.Y, t, PPP);               // Y3 = R(Q - X3) - S1 PPP
+  }
+
+  // XYZZ (Montgomery) -> canonical affine, O -> (0,0).
+  GZ_DEV static void to_affine_canonical(uint32_t x[N], uint32_t y[N], const Xyzz& P) {
+    if (is_inf(P)) { Fp::set_zero(x); Fp::set_zero(y); return; }
+    uint32_t d[N], inv[N], t[N];
+    Fp::mul(d, P.ZZ, P.ZZZ);
+    Fp::inv(inv, d);                    // 1 / (ZZ ZZZ)
+    Fp::mul(t, inv, P.ZZZ);             // 1 / ZZ
+    Fp::mul(t, P.X, t);
+    Fp::from_mont(x, t);
+    Fp::mul(t, inv, P.ZZ);              // 1 / ZZZ
+    Fp::mul(t, P.Y, t);
+    Fp::from_mont(y, t);
+  }
+
+  // vectorised copies of one N-limb coordinate (16-B aligned when N % 4 == 0)
+  GZ_DEV static void ld(uint32_t d[N], const uint32_t* src) {
+    if constexpr (N % 4 == 0) {
+      const uint4* s = reinterpret_cast<const uint4*>(src);
+#pragma unroll
+      for (int i = 0; i < N / 4; ++i) {
+        uint4 v = s[i];
+        d[4 * i] = v.x; d[4 * i + 1] = v.y; d[4 * i + 2] = v.z; d[4 * i + 3] = v.w;
+      }
+    } else {
+      const uint2* s = reinterpret_cast<const uint2*>(src);
+#pragma unroll
+      for (int i = 0; i < N / 2; ++i) { uint2 v = s[i]; d[2 * i] = v.x; d[2 * i + 1] = v.y; }
+    }
+  }
+  GZ_DEV static void st(uint32_t* dst, const uint32_t d[N]) {
+    if constexpr (N % 4 == 0) {
+      uint4* s = reinterpret_cast<uint4*>(dst);
+#pragma unroll
+      for (int i = 0; i < N / 4; ++i) s[i] = make_uint4(d[4 * i], d[4 * i + 1], d[4 * i + 2], d[4 * i + 3]);
+    } else {
+      uint2* s = reinterpret_cast<uint2*>(dst);
+#pragma unroll
+      for (int i = 0; i < N / 2; ++i) s[i] = make_uint2(d[2 * i], d[2 * i + 1]);
+    }
+  }
+  // an XYZZ point in memory is X || Y || ZZ || ZZZ (4N u32, Montgomery form)
+  GZ_DEV static void load(Xyzz& P, const uint32_t* src) {
+    ld(P.X, src); ld(P.Y, src + N); ld(P.ZZ, src + 2 * N); ld(P.ZZZ, src + 3 * N);
+  }
+  GZ_DEV static void store(uint32_t* dst, const Xyzz& P) {
+    st(dst, P.X); st(dst + N, P.Y); st(dst + 2 * N, P.ZZ); st(dst + 3 * N, P.ZZZ);
+  }
+};
+
+// ---- out-of-line versions for the cold kernels (merge, reduction, tail,
+// generators, diagnostics): one copy of each group-law body per TU keeps the
+// compile time and the instruction footprint bounded; only the bucket hot loop
+// (k_accum) inlines madd.
+template <class C>
+__device__ __noinline__ void ec_add(typename EC<C>::Xyzz& A, const typename EC<C>::Xyzz& B) { EC<C>::add(A, B); }
+template <class C>
+__device__ __noinline__ void ec_dbl(typename EC<C>::Xyzz& A) { EC<C>::dbl(A); }
+template <class C>
+__device__ __noinline__ void ec_madd(typename EC<C>::Xyzz& A, const uint32_t* x, const uint32_t* y) {
+  uint32_t xx[C::N], yy[C::N];
+#pragma unroll
+  for (int i = 0; i < C::N; ++i) { xx[i] = x[i]; yy[i] = y[i]; }
+  EC<C>::madd_nz(A, xx, yy);
+}
+template <class C>
+__device__ __noinline__ void ec_mdbl(typename EC<C>::Xyzz& A, const uint32_t* x, const uint32_t* y) {
+  uint32_t xx[C::N], yy[C::N];
+#pragma unroll
+  for (int i = 0; i < C::N; ++i) { xx[i] = x[i]; yy[i] = y[i]; }
+  EC<C>::mdbl(A, xx, yy);
+}
+template <class C>
+__device__ __noinline__ void ec_to_affine(uint32_t* x, uint32_t* y, const typename EC<C>::Xyzz& P) {
+  uint32_t xx[C::N], yy[C::N];
+  EC<C>::to_affine_canonical(xx, yy, P);
+#pragma unroll
+  for (int i = 0; i < C::N; ++i) { x[i] = xx[i]; y[i] = yy[i]; }
+}
+// P = k * P for a small non-negative integer k (double-and-add, MSB first)
+template <class C>
+__device__ __noinline__ void ec_mul_small(typename EC<C>::Xyzz& P, uint32_t k) {
+  using E = EC<C>;
+  if (k == 0 || E::is_inf(P)) { E::set_inf(P); return; }
+  typename E::Xyzz B = P;
+  const int top = 31 - __clz(k);
+  for (int i = top - 1; i >= 0; --i) {
+    ec_dbl<C>(P);
+    if ((k >> i) & 1) ec_add<C>(P, B);
+  }
+}
+
+}  // namespace gzkp

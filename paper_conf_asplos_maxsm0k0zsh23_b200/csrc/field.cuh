@@ -1,0 +1,290 @@
+// field.cuh -- multi-limb Montgomery arithmetic over F_p on 32-bit IMAD carry chains.
+//
+// The paper's finite-field library (§4.3) multiplies big
+// integers with "modular multiplications [52]" (Montgomery) on
+// 64-bit words split across cooperating threads, plus a DFP/FP64 path.  On
+// sm_100 there is no 64-bit integer multiplier: the native unit is the 32-bit
+// IMAD (lo / hi halves, with hardware carry-in/out), so one thread holds one
+// element as N little-endian u32 limbs in registers (N = 8 / 12 / 24) and the
+// product uses the CIOS schedule with the multiplicand split into even and odd
+// limbs: a[2j]*b_i lands on limb pairs (2j, 2j+1) and a[2j+1]*b_i on
+// (2j+1, 2j+2), so each half is ONE unbroken mad.lo.cc / madc.hi.cc chain.
+// Two independent chains per row give the scheduler ILP.  The accumulators swap
+// roles each row so the shift by one limb costs no moves
+// (tools/emulate_mont.py checks the sequence carry-exactly).
+//
+// Cost: mont_mul = N(4N+1) IMAD (264 / 588 / 2328 for N = 8 / 12 / 24).
+// Values are kept fully reduced in [0, p): the group law's equality tests
+// (madd's U2 == X1) need canonical representatives.
+#pragma once
+#include <cstdint>
+
+namespace gzkp {
+
+#define GZ_DEV __device__ __forceinline__
+
+// ---------------------------------------------------------------- PTX glue
+// Each helper is one instruction; the carry flag (CC) flows between
+// consecutive asm volatile statements exactly as written.
+GZ_DEV uint32_t mul_lo(uint32_t a, uint32_t b) { uint32_t r; asm("mul.lo.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b)); return r; }
+GZ_DEV uint32_t mul_hi(uint32_t a, uint32_t b) { uint32_t r; asm("mul.hi.u32 %0, %1, %2;" : "=r"(r) : "r"(a), "r"(b)); return r; }
+
+#define MAD_LO_CC(d, a, b, c)   asm volatile("mad.lo.cc.u32 %0, %1, %2, %3;"  : "=r"(d) : "r"(a), "r"(b), "r"(c))
+#define MADC_LO_CC(d, a, b, c)  asm volatile("madc.lo.cc.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c))
+#define MADC_HI_CC(d, a, b, c)  asm volatile("madc.hi.cc.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(b), "r"(c))
+#define MADC_HI(d, a, b, c)     asm volatile("madc.hi.u32 %0, %1, %2, %3;"    : "=r"(d) : "r"(a), "r"(b), "r"(c))
+#define ADD_CC(d, a, b)         asm volatile("add.cc.u32 %0, %1, %2;"  : "=r"(d) : "r"(a), "r"(b))
+#define ADDC_CC(d, a, b)        asm volatile("addc.cc.u32 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b))
+#define ADDC(d, a, b)           asm volatile("addc.u32 %0, %1, %2;"    : "=r"(d) : "r"(a), "r"(b))
+#define SUB_CC(d, a, b)         asm volatile("sub.cc.u32 %0, %1, %2;"  : "=r"(d) : "r"(a), "r"(b))
+#define SUBC_CC(d, a, b)        asm volatile("subc.cc.u32 %0, %1, %2;" : "=r"(d) : "r"(a), "r"(b))
+#define SUBC(d, a, b)           asm volatile("subc.u32 %0, %1, %2;"    : "=r"(d) : "r"(a), "r"(b))
+
+// ------------------------------------------------------- F_p element ops
+// All functions take/return arrays of C::N u32 limbs (registers after unroll).
+
+template <class C>
+struct F {
+  static constexpr int N = C::N;
+
+  GZ_DEV static void copy(uint32_t r[N], const uint32_t a[N]) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) r[i] = a[i];
+  }
+  GZ_DEV static void set_zero(uint32_t r[N]) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) r[i] = 0;
+  }
+  GZ_DEV static void set_one(uint32_t r[N]) {   // Montgomery 1 = R mod p
+#pragma unroll
+    for (int i = 0; i < N; ++i) r[i] = C::ONE(i);
+  }
+  GZ_DEV static bool is_zero(const uint32_t a[N]) {
+    uint32_t t = a[0];
+#pragma unroll
+    for (int i = 1; i < N; ++i) t |= a[i];
+    return t == 0;
+  }
+  GZ_DEV static bool eq(const uint32_t a[N], const uint32_t b[N]) {
+    uint32_t t = a[0] ^ b[0];
+#pragma unroll
+    for (int i = 1; i < N; ++i) t |= a[i] ^ b[i];
+    return t == 0;
+  }
+
+  // r = a - p if a >= p (a < 2p, and a fits in N limbs: p has spare bits)
+  GZ_DEV static void reduce_once(uint32_t a[N]) {
+    uint32_t t[N], borrow;
+    SUB_CC(t[0], a[0], C::P(0));
+#pragma unroll
+    for (int i = 1; i < N; ++i) SUBC_CC(t[i], a[i], C::P(i));
+    SUBC(borrow, 0u, 0u);          // 0 if a >= p, 0xffffffff otherwise
+#pragma unroll
+    for (int i = 0; i < N; ++i) a[i] = borrow ? a[i] : t[i];
+  }
+
+  // r = a + b mod p
+  GZ_DEV static void add(uint32_t r[N], const uint32_t a[N], const uint32_t b[N]) {
+    ADD_CC(r[0], a[0], b[0]);
+#pragma unroll
+    for (int i = 1; i < N - 1; ++i) ADDC_CC(r[i], a[i], b[i]);
+    ADDC(r[N - 1], a[N - 1], b[N - 1]);   // no overflow: p < 2^(32N - 1)
+    reduce_once(r);
+  }
+
+  // r = a - b mod p
+  GZ_DEV static void sub(uint32_t r[N], const uint32_t a[N], const uint32_t b[N]) {
+    uint32_t borrow, t[N];
+    SUB_CC(r[0], a[0], b[0]);
+#pragma unroll
+    for (int i = 1; i < N; ++i) SUBC_CC(r[i], a[i], b[i]);
+    SUBC(borrow, 0u, 0u);          // 0xffffffff if a < b
+#pragma unroll
+    for (int i = 0; i < N; ++i) t[i] = C::P(i) & borrow;
+    ADD_CC(r[0], r[0], t[0]);
+#pragma unroll
+    for (int i = 1; i < N - 1; ++i) ADDC_CC(r[i], r[i], t[i]);
+    ADDC(r[N - 1], r[N - 1], t[N - 1]);
+  }
+
+  GZ_DEV static void dbl(uint32_t r[N], const uint32_t a[N]) { add(r, a, a); }
+
+  // r = -a mod p
+  GZ_DEV static void neg(uint32_t r[N], const uint32_t a[N]) {
+    uint32_t z[N];
+    set_zero(z);
+    sub(r, z, a);
+  }
+
+  // ---- Montgomery product r = a * b * R^-1 mod p (even/odd CIOS) ----
+  // E holds limbs at positions 0..N-1, O at positions 1..N (one limb up).
+  // For N >= 24 (MNT4-753) the product is an out-of-line call: a fully inlined
+  // 2328-IMAD body at every call site makes the kernels too large to compile.
+  GZ_DEV static void mul(uint32_t r[N], const uint32_t a[N], const uint32_t b[N]) {
+    if constexpr (N >= 24) mul_ni(r, a, b);
+    else mul_inline(r, a, b);
+  }
+  __device__ __noinline__ static void mul_ni(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+    uint32_t x[N], y[N], z[N];
+#pragma unroll
+    for (int i = 0; i < N; ++i) { x[i] = a[i]; y[i] = b[i]; }
+    mul_inline(z, x, y);
+#pragma unroll
+    for (int i = 0; i < N; ++i) r[i] = z[i];
+  }
+  GZ_DEV static void mul_inline(uint32_t r[N], const uint32_t a[N], const uint32_t b[N]) {
+    uint32_t e[N], o[N];
+    uint32_t* E = e;
+    uint32_t* O = o;
+    // row 0: plain products
+    {
+      const uint32_t bi = b[0];
+#pragma unroll
+      for (int j = 0; j < N; j += 2) {
+        E[j] = mul_lo(a[j], bi);
+        E[j + 1] = mul_hi(a[j], bi);
+        O[j] = mul_lo(a[j + 1], bi);
+        O[j + 1] = mul_hi(a[j + 1], bi);
+      }
+      redc_step(E, O);
+    }
+#pragma unroll
+    for (int i = 1; i < N; ++i) {
+      uint32_t* t = E; E = O; O = t;      // roles swap (compile-time after unroll)
+      const uint32_t bi = b[i];
+      // E[0] += O_old_shifted[1]; carry flows into the O chain at position 1
+      ADD_CC(E[0], E[0], O[1]);
+      // O_new[k] = a_odd * bi + O_old[k + 2]   (the one-limb shift)
+#pragma unroll
+      for (int j = 0; j < N - 2; j += 2) {
+        MADC_LO_CC(O[j], a[j + 1], bi, O[j + 2]);
+        MADC_HI_CC(O[j + 1], a[j + 1], bi, O[j + 3]);
+      }
+      MADC_LO_CC(O[N - 2], a[N - 1], bi, 0u);
+      MADC_HI(O[N - 1], a[N - 1], bi, 0u);
+      // E += a_even * bi, top carry into O[N-1] (position N)
+      MAD_LO_CC(E[0], a[0], bi, E[0]);
+      MADC_HI_CC(E[1], a[0], bi, E[1]);
+#pragma unroll
+      for (int j = 2; j < N; j += 2) {
+        MADC_LO_CC(E[j], a[j], bi, E[j]);
+        MADC_HI_CC(E[j + 1], a[j], bi, E[j + 1]);
+      }
+      ADDC(O[N - 1], O[N - 1], 0u);
+      redc_step(E, O);
+    }
+    // r = (E >> 32) + O
+    ADD_CC(r[0], E[1], O[0]);
+#pragma unroll
+    for (int k = 1; k < N - 1; ++k) ADDC_CC(r[k], E[k + 1], O[k]);
+    ADDC(r[N - 1], O[N - 1], 0u);
+    reduce_once(r);
+  }
+
+  // m = E[0] * n0; E += m * p_even; O += m * p_odd  (makes E[0] == 0)
+  GZ_DEV static void redc_step(uint32_t* E, uint32_t* O) {
+    const uint32_t m = E[0] * C::N0;
+    MAD_LO_CC(O[0], C::P(1), m, O[0]);
+    MADC_HI_CC(O[1], C::P(1), m, O[1]);
+#pragma unroll
+    for (int j = 2; j < N - 2; j += 2) {
+      MADC_LO_CC(O[j], C::P(j + 1), m, O[j]);
+      MADC_HI_CC(O[j + 1], C::P(j + 1), m, O[j + 1]);
+    }
+    if (N > 2) {
+      MADC_LO_CC(O[N - 2], C::P(N - 1), m, O[N - 2]);
+      MADC_HI(O[N - 1], C::P(N - 1), m, O[N - 1]);
+    }
+    MAD_LO_CC(E[0], C::P(0), m, E[0]);
+    MADC_HI_CC(E[1], C::P(0), m, E[1]);
+#pragma unroll
+    for (int j = 2; j < N; j += 2) {
+      MADC_LO_CC(E[j], C::P(j), m, E[j]);
+      MADC_HI_CC(E[j + 1], C::P(j), m, E[j + 1]);
+    }
+    ADDC(O[N - 1], O[N - 1], 0u);
+  }
+
+  GZ_DEV static void sqr(uint32_t r[N], const uint32_t a[N]) { mul(r, a, a); }
+
+  GZ_DEV static void to_mont(uint32_t r[N], const uint32_t a[N]) {
+    uint32_t r2[N];
+#pragma unroll
+    for (int i = 0; i < N; ++i) r2[i] = C::R2(i);
+    mul(r, a, r2);
+  }
+  GZ_DEV static void from_mont(uint32_t r[N], const uint32_t a[N]) {
+    uint32_t one[N];
+    set_zero(one);
+    one[0] = 1;
+    mul(r, a, one);
+  }
+
+  // ---- inverse of a CANONICAL (non-Montgomery) value by binary extended
+  // Euclid; a != 0.  Latency ~2*bits iterations of N-limb shifts/subtracts,
+  // far shorter than Fermat's ~1.5*bits serial multiplications.
+  GZ_DEV static void shr1(uint32_t x[N], uint32_t top) {
+#pragma unroll
+    for (int i = 0; i < N - 1; ++i) x[i] = __funnelshift_r(x[i], x[i + 1], 1);
+    x[N - 1] = (x[N - 1] >> 1) | (top << 31);
+  }
+  GZ_DEV static void half_mod(uint32_t x[N]) {   // x/2 mod p for x in [0, p)
+    if (x[0] & 1) {
+      uint32_t c;
+      ADD_CC(x[0], x[0], C::P(0));
+#pragma unroll
+      for (int i = 1; i < N; ++i) ADDC_CC(x[i], x[i], C::P(i));
+      ADDC(c, 0u, 0u);
+      shr1(x, c);
+    } else {
+      shr1(x, 0);
+    }
+  }
+  GZ_DEV static bool is_one_int(const uint32_t a[N]) {
+    uint32_t t = a[0] ^ 1u;
+#pragma unroll
+    for (int i = 1; i < N; ++i) t |= a[i];
+    return t == 0;
+  }
+  // returns borrow (a < b) and r = a - b (integer)
+  GZ_DEV static bool sub_int(uint32_t r[N], const uint32_t a[N], const uint32_t b[N]) {
+    uint32_t borrow;
+    SUB_CC(r[0], a[0], b[0]);
+#pragma unroll
+    for (int i = 1; i < N; ++i) SUBC_CC(r[i], a[i], b[i]);
+    SUBC(borrow, 0u, 0u);
+    return borrow != 0;
+  }
+  GZ_DEV static void inv_canonical(uint32_t r[N], const uint32_t a[N]) {
+    uint32_t u[N], v[N], x1[N], x2[N], t[N];
+    copy(u, a);
+#pragma unroll
+    for (int i = 0; i < N; ++i) v[i] = C::P(i);
+    set_zero(x1);
+    x1[0] = 1;
+    set_zero(x2);
+    if (is_zero(a)) { set_zero(r); return; }   // no inverse; never loop forever
+    // each outer pass strips >= 1 bit from u or v: <= 2 * 32N passes
+    for (int guard = 0; guard < 64 * N + 8 && !is_one_int(u) && !is_one_int(v); ++guard) {
+      while (!(u[0] & 1)) { shr1(u, 0); half_mod(x1); }
+      while (!(v[0] & 1)) { shr1(v, 0); half_mod(x2); }
+      if (!sub_int(t, u, v)) {       // u >= v
+        copy(u, t);
+        sub(x1, x1, x2);
+      } else {
+        sub_int(v, v, u);
+        sub(x2, x2, x1);
+      }
+    }
+    if (is_one_int(u)) copy(r, x1); else copy(r, x2);
+  }
+  // Montgomery-domain inverse: (aR)^-1 R = from/to conversions around EEA
+  GZ_DEV static void inv(uint32_t r[N], const uint32_t a[N]) {
+    uint32_t c[N], ic[N];
+    from_mont(c, a);
+    inv_canonical(ic, c);
+    to_mont(r, ic);
+  }
+};
+
+}  // namespace gzkp

@@ -1,0 +1,73 @@
+// internal.h -- interface between the C ABI (abi.cu) and the per-curve
+// template instantiations (curve_*.cu).  Not part of the public ABI.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstddef>
+#include <cstdint>
+#include <string>
+
+#include "../../include/gzkp.h"
+
+namespace gzkp {
+
+inline size_t align_up(size_t x, size_t a = 256) { return (x + a - 1) / a * a; }
+
+struct Tunables {
+  int window_bits = 0;     // 0 = cost model
+  int chunk_entries = 0;   // 0 = default
+};
+Tunables& tunables();
+
+// one MSM invocation (device pointers)
+struct MsmCall {
+  const void* points = nullptr;   // canonical affine, or Montgomery when prepared
+  bool prepared = false;
+  const void* scalars = nullptr;
+  size_t n = 0;
+  void* out_affine = nullptr;     // canonical affine result (may be null)
+  void* out_partial = nullptr;    // XYZZ partial (may be null)
+  void* workspace = nullptr;      // null = stream-ordered allocation inside
+  size_t workspace_bytes = 0;
+  cudaStream_t stream = nullptr;
+};
+
+struct CurveImpl {
+  int id;
+  int limbs;          // N
+  int scalar_limbs;   // NS
+  int scalar_bits;
+  int (*window_bits)(size_t n);
+  size_t (*workspace_bytes)(size_t n, bool prepared);
+  gzkp_status (*msm)(const MsmCall& call);
+  gzkp_status (*to_mont)(const void* in, void* out, size_t n, cudaStream_t s);
+  gzkp_status (*combine)(const void* partials, int count, void* out, cudaStream_t s);
+  gzkp_status (*fixed_base)(const void* scalars, size_t n, void* out, cudaStream_t s);
+  gzkp_status (*field_op)(int op, const void* a, const void* b, void* out, size_t n, cudaStream_t s);
+  gzkp_status (*ec_op)(int op, const void* P, const void* Q, void* out, size_t n, cudaStream_t s);
+};
+
+const CurveImpl* impl_bn254();
+const CurveImpl* impl_bls12_381();
+const CurveImpl* impl_mnt4_753();
+const CurveImpl* impl_toy_a0();
+const CurveImpl* impl_toy_a2();
+const CurveImpl* impl_for(int curve);
+
+gzkp_status set_error(gzkp_status st, const std::string& msg);
+gzkp_status cuda_status(cudaError_t e, const char* where);
+int device_sm_count();
+bool profiling_enabled();
+// profiling hooks (no synchronisation): events[6] recorded by the caller,
+// entries_dev = device address of the call's entry count (copied async).
+struct ProfileRecord {
+  cudaEvent_t ev[6];
+  uint32_t* entries_host;   // pinned, written by an async copy
+  int launches;
+  int c;
+};
+ProfileRecord* profile_begin(cudaStream_t s);          // null when profiling is off
+void profile_mark(ProfileRecord* r, int i, cudaStream_t s);
+void profile_end(ProfileRecord* r, const uint32_t* entries_dev, int launches, int c, cudaStream_t s);
+
+}  // namespace gzkp

@@ -1,0 +1,607 @@
+// msm_kernels.cuh -- the Pippenger pipeline kernels (one template per curve).
+//
+// Steps:
+//   a1 k_to_mont       canonical affine -> Montgomery affine        ("P ... unchanged")
+//   a2 k_hist          signed c-bit digits -> per-window bucket histogram
+//      k_scan_*        exclusive scan -> bucket offsets
+//   a3 k_scatter       counting-sort scatter of (bucket key, point idx|sign)  (p_index)
+//   a4 k_accum         equal-work chunks of the sorted entries, XYZZ madd hot loop,
+//                      points staged in shared memory by cp.async
+//   a5 k_merge         level-wise segmented reduction of chunk-boundary partials
+//   a6 k_reduce_seg/_win  bucket reduction sum_j j*B_j by running sums
+//   a7 k_tail          window combination sum_t 2^(ct) W_t (Horner)
+//   a8 k_tail/k_combine   normalise XYZZ -> canonical affine
+#pragma once
+#include <cuda_runtime.h>
+
+#include "ec.cuh"
+
+namespace gzkp {
+
+constexpr uint32_t KEY_REAL = 0x80000000u;   // slot key flag: payload present
+constexpr uint32_t VAL_NEG = 0x80000000u;    // entry flag: negative digit
+constexpr uint32_t KEY_NONE = 0xffffffffu;
+
+// Per-level device counters written by k_plan (all derived from E on device).
+struct LevelInfo {
+  uint32_t E;            // total entries (non-zero digits)
+  uint32_t n[40];        // n[0] = chunks at level 0; n[l] (l>=1) = slots input to merge level l
+};
+
+// ---------------------------------------------------------------- digits
+// Booth-style signed recoding: d_t = v_t + k_{ct-1} - 2^c * k_{ct+c-1}, with
+// v_t = bits [ct, ct+c) of k.  Each digit depends only on c+1 bits, so windows
+// are independent; d_t in [-2^(c-1), 2^(c-1)] and sum_t d_t 2^(ct) = k when
+// k < 2^(cW-1), i.e. W = ceil((b+1)/c) (reading R7).
+template <int NS>
+GZ_DEV int booth_digit(const uint32_t* __restrict__ k, int t, int c) {
+  const int pos = t * c - 1;
+  uint32_t x;
+  if (pos < 0) {
+    x = (__ldg(k) << 1);
+  } else {
+    const int w = pos >> 5, off = pos & 31;
+    const uint32_t lo = w < NS ? __ldg(k + w) : 0u;
+    const uint32_t hi = (w + 1) < NS ? __ldg(k + w + 1) : 0u;
+    x = __funnelshift_r(lo, hi, off);
+  }
+  x &= (c >= 31) ? 0xffffffffu : ((2u << c) - 1u);
+  return (int)(x >> 1) + (int)(x & 1u) - (int)(((x >> c) & 1u) << c);
+}
+
+// ------------------------------------------------------------ a1 to_mont
+template <class C>
+__global__ void k_to_mont(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, size_t n) {
+  using Fp = F<C>;
+  using E = EC<C>;
+  constexpr int N = C::N;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    uint32_t x[N], y[N];
+    E::ld(x, in + i * 2 * N);
+    E::ld(y, in + i * 2 * N + N);
+    Fp::to_mont(x, x);
+    Fp::to_mont(y, y);
+    E::st(out + i * 2 * N, x);
+    E::st(out + i * 2 * N + N, y);
+  }
+}
+
+// --------------------------------------------------- a2 histogram (smem)
+// grid = (blocks_per_window, W); block (bx, t) counts window t's digits of
+// points [bx*per, ...) in a shared-memory histogram of B bins, then flushes
+// the non-zero bins with one global atomic each.  Skewed inputs (the sparse
+// witness's bucket 1) contend only in shared memory.
+template <class C>
+__global__ void k_hist(const uint32_t* __restrict__ sc, size_t n, int c, uint32_t B,
+                       uint32_t* __restrict__ counts) {
+  extern __shared__ uint32_t hist[];
+  const int t = blockIdx.y;
+  for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
+  __syncthreads();
+  const size_t per = (n + gridDim.x - 1) / gridDim.x;
+  const size_t beg = blockIdx.x * per, end = min(n, beg + per);
+  for (size_t i = beg + threadIdx.x; i < end; i += blockDim.x) {
+    const int d = booth_digit<C::NS>(sc + i * C::NS, t, c);
+    if (d) atomicAdd(&hist[abs(d) - 1], 1u);
+  }
+  __syncthreads();
+  for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
+    const uint32_t h = hist[b];
+    if (h) atomicAdd(&counts[(size_t)t * B + b], h);
+  }
+}
+
+// ----------------------------------------------------- scan (exclusive)
+constexpr int SCAN_THREADS = 1024;
+constexpr int SCAN_PER_THREAD = 4;
+constexpr int SCAN_TILE = SCAN_THREADS * SCAN_PER_THREAD;
+
+GZ_DEV uint32_t block_exclusive_scan(uint32_t v, uint32_t* warp_sums, uint32_t* total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) warp_sums[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    uint32_t s = lane < (int)(blockDim.x >> 5) ? warp_sums[lane] : 0u;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(0xffffffffu, s, o);
+      if (lane >= o) s += y;
+    }
+    warp_sums[lane] = s;    // inclusive
+  }
+  __syncthreads();
+  const uint32_t base = wid ? warp_sums[wid - 1] : 0u;
+  if (total) *total = warp_sums[(blockDim.x >> 5) - 1];
+  return base + x - v;
+}
+
+static __global__ void k_scan_tiles(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, uint32_t M,
+                             uint32_t* __restrict__ tile_sums) {
+  __shared__ uint32_t ws[32];
+  const size_t base = (size_t)blockIdx.x * SCAN_TILE + threadIdx.x * SCAN_PER_THREAD;
+  uint32_t v[SCAN_PER_THREAD], s = 0;
+#pragma unroll
+  for (int k = 0; k < SCAN_PER_THREAD; ++k) {
+    v[k] = (base + k < M) ? in[base + k] : 0u;
+    s += v[k];
+  }
+  uint32_t total;
+  uint32_t ex = block_exclusive_scan(s, ws, &total);
+#pragma unroll
+  for (int k = 0; k < SCAN_PER_THREAD; ++k) {
+    if (base + k < M) out[base + k] = ex;
+    ex += v[k];
+  }
+  if (threadIdx.x == 0) tile_sums[blockIdx.x] = total;
+}
+
+// single block: exclusive scan of tile sums (<= SCAN_TILE tiles), writes total to out_total
+static __global__ void k_scan_top(uint32_t* __restrict__ tile_sums, uint32_t ntiles, uint32_t* __restrict__ out_total) {
+  __shared__ uint32_t ws[32];
+  const uint32_t base = threadIdx.x * SCAN_PER_THREAD;
+  uint32_t v[SCAN_PER_THREAD], s = 0;
+#pragma unroll
+  for (int k = 0; k < SCAN_PER_THREAD; ++k) {
+    v[k] = (base + k < ntiles) ? tile_sums[base + k] : 0u;
+    s += v[k];
+  }
+  uint32_t total;
+  uint32_t ex = block_exclusive_scan(s, ws, &total);
+#pragma unroll
+  for (int k = 0; k < SCAN_PER_THREAD; ++k) {
+    if (base + k < ntiles) tile_sums[base + k] = ex;
+    ex += v[k];
+  }
+  if (threadIdx.x == 0) *out_total = total;
+}
+
+static __global__ void k_scan_add(uint32_t* __restrict__ out, uint32_t* __restrict__ cursor, uint32_t M,
+                           const uint32_t* __restrict__ tile_sums) {
+  const uint32_t add = tile_sums[blockIdx.x];
+  const size_t base = (size_t)blockIdx.x * SCAN_TILE;
+  for (uint32_t k = threadIdx.x; k < SCAN_TILE; k += blockDim.x) {
+    if (base + k < M) {
+      const uint32_t v = out[base + k] + add;
+      out[base + k] = v;
+      cursor[base + k] = v;
+    }
+  }
+}
+
+// ------------------------------------------------------------ plan counts
+static __global__ void k_plan(const uint32_t* __restrict__ offsets, uint32_t M, int S, int S2, int levels,
+                       LevelInfo* __restrict__ info) {
+  if (threadIdx.x || blockIdx.x) return;
+  const uint32_t E = offsets[M];
+  info->E = E;
+  uint32_t chunks = (E + S - 1) / S;
+  info->n[0] = chunks;
+  uint32_t slots = 2 * chunks;
+  for (int l = 1; l <= levels && l < 40; ++l) {
+    info->n[l] = slots;
+    slots = 2 * ((slots + S2 - 1) / S2);
+  }
+}
+
+// ------------------------------------------------------- a3 scatter (sort)
+// Same grid as k_hist.  Block-local counts are reserved in the global bucket
+// ranges with one atomic per non-zero bin; entries then take consecutive
+// positions from a shared-memory cursor.
+template <class C>
+__global__ void k_scatter(const uint32_t* __restrict__ sc, size_t n, int c, uint32_t B,
+                          uint32_t* __restrict__ cursor, uint32_t* __restrict__ keys,
+                          uint32_t* __restrict__ vals) {
+  extern __shared__ uint32_t hist[];
+  const int t = blockIdx.y;
+  for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
+  __syncthreads();
+  const size_t per = (n + gridDim.x - 1) / gridDim.x;
+  const size_t beg = blockIdx.x * per, end = min(n, beg + per);
+  for (size_t i = beg + threadIdx.x; i < end; i += blockDim.x) {
+    const int d = booth_digit<C::NS>(sc + i * C::NS, t, c);
+    if (d) atomicAdd(&hist[abs(d) - 1], 1u);
+  }
+  __syncthreads();
+  for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
+    const uint32_t h = hist[b];
+    hist[b] = h ? atomicAdd(&cursor[(size_t)t * B + b], h) : 0u;
+  }
+  __syncthreads();
+  const uint32_t kbase = (uint32_t)t * B;
+  for (size_t i = beg + threadIdx.x; i < end; i += blockDim.x) {
+    const int d = booth_digit<C::NS>(sc + i * C::NS, t, c);
+    if (d) {
+      const uint32_t b = abs(d) - 1;
+      const uint32_t pos = atomicAdd(&hist[b], 1u);
+      keys[pos] = kbase + b;
+      vals[pos] = (uint32_t)i | (d < 0 ? VAL_NEG : 0u);
+    }
+  }
+}
+
+// ---------------------------------------------------------- cp.async glue
+GZ_DEV void cp_async16(void* smem, const void* gmem) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+GZ_DEV void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int K>
+GZ_DEV void cp_async_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(K) : "memory"); }
+
+template <class C>
+struct Stage {
+  static constexpr int N = C::N;
+  static constexpr int PT_WORDS = 2 * N;                 // one affine point
+  static constexpr int SLOT_WORDS = 2 * PT_WORDS + 4;    // double buffer + 16 B pad (bank spread)
+  static constexpr int PT_CHUNKS = PT_WORDS / 4;         // 16-B pieces per point
+  GZ_DEV static void fetch(uint32_t* slot_buf, const uint32_t* __restrict__ pts, uint32_t idx) {
+    const uint32_t* src = pts + (size_t)idx * PT_WORDS;
+#pragma unroll
+    for (int q = 0; q < PT_CHUNKS; ++q) cp_async16(slot_buf + 4 * q, src + 4 * q);
+  }
+};
+
+// -------------------------------------------------- a4 bucket accumulation
+// Persistent grid-stride loop over chunks of S consecutive sorted entries.  A
+// chunk may cut through buckets: runs that lie wholly inside the chunk are
+// written straight to their bucket; a run touching the chunk boundary (its
+// bucket continues in the neighbouring chunk) becomes a "boundary partial" in
+// slot 2*chunk (first run) or 2*chunk+1 (last run) for the merge levels.
+// Unused slots carry the chunk's first / last key as a payload-less dummy so
+// the slot keys stay sorted.
+template <class C>
+__global__ void __launch_bounds__(128) k_accum(const uint32_t* __restrict__ keys, const uint32_t* __restrict__ vals,
+                                               const uint32_t* __restrict__ pts, const LevelInfo* __restrict__ info,
+                                               int S, uint32_t* __restrict__ buckets,
+                                               uint32_t* __restrict__ skeys, uint32_t* __restrict__ spay) {
+  using Fp = F<C>;
+  using EC_ = EC<C>;
+  using St = Stage<C>;
+  constexpr int N = C::N;
+  extern __shared__ __align__(16) uint32_t stage_smem[];
+  uint32_t* slot = stage_smem + threadIdx.x * St::SLOT_WORDS;
+
+  const uint32_t E = info->E;
+  const uint32_t nchunks = info->n[0];
+  for (uint32_t chunk = blockIdx.x * blockDim.x + threadIdx.x; chunk < nchunks;
+       chunk += gridDim.x * blockDim.x) {
+    const uint32_t beg = chunk * (uint32_t)S;
+    const uint32_t end = min(E, beg + (uint32_t)S);
+    const uint32_t prev_key = beg ? keys[beg - 1] : KEY_NONE;
+    const uint32_t next_key = end < E ? keys[end] : KEY_NONE;
+    const uint32_t first_key = keys[beg];
+    const uint32_t last_key = keys[end - 1];
+    bool head_written = false, tail_written = false;
+
+    typename EC_::Xyzz acc;
+    bool acc_inf = true;
+    uint32_t cur = first_key;
+    bool first_run = true;
+
+    auto flush = [&](bool last_run) {
+      const bool open_l = first_run && prev_key == cur;
+      const bool open_r = last_run && next_key == cur;
+      if (acc_inf) EC_::set_inf(acc);
+      if (!open_l && !open_r) {
+        EC_::store(buckets + (size_t)cur * 4 * N, acc);
+      } else {
+        const uint32_t s = open_l ? 2 * chunk : 2 * chunk + 1;
+        skeys[s] = cur | KEY_REAL;
+        EC_::store(spay + (size_t)s * 4 * N, acc);
+        if (open_l) head_written = true; else tail_written = true;
+      }
+    };
+
+    uint32_t v_next = vals[beg];
+    St::fetch(slot, pts, v_next & ~VAL_NEG);
+    cp_async_commit();
+    for (uint32_t j = beg; j < end; ++j) {
+      const uint32_t key = keys[j];
+      const uint32_t v = v_next;
+      const int buf = (j - beg) & 1;
+      if (j + 1 < end) {
+        v_next = vals[j + 1];
+        St::fetch(slot + (buf ^ 1) * St::PT_WORDS, pts, v_next & ~VAL_NEG);
+      }
+      cp_async_commit();
+      cp_async_wait<1>();
+      if (key != cur) {
+        flush(false);
+        acc_inf = true;
+        cur = key;
+        first_run = false;
+      }
+      uint32_t x[N], y[N];
+      EC_::ld(x, slot + buf * St::PT_WORDS);
+      EC_::ld(y, slot + buf * St::PT_WORDS + N);
+      if (Fp::is_zero(x) && Fp::is_zero(y)) continue;     // identity input point
+      if (v & VAL_NEG) Fp::neg(y, y);
+      if (acc_inf) {
+        EC_::from_affine(acc, x, y);
+        acc_inf = false;
+      } else {
+        EC_::madd_nz(acc, x, y);
+        acc_inf = EC_::is_inf(acc);
+      }
+    }
+    cp_async_wait<0>();
+    flush(true);
+    if (!head_written) skeys[2 * chunk] = first_key;
+    if (!tail_written) skeys[2 * chunk + 1] = last_key;
+  }
+}
+
+// --------------------------------------------------------- a5 merge level
+// Same run logic over slots (key|REAL, XYZZ payload) with the full XYZZ add.
+template <class C>
+__global__ void __launch_bounds__(128) k_merge(const uint32_t* __restrict__ in_keys, const uint32_t* __restrict__ in_pay,
+                                               const LevelInfo* __restrict__ info, int level, int S2,
+                                               uint32_t* __restrict__ buckets, uint32_t* __restrict__ out_keys,
+                                               uint32_t* __restrict__ out_pay) {
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  const uint32_t n_in = info->n[level];
+  const uint32_t nchunks = (n_in + S2 - 1) / S2;
+  for (uint32_t chunk = blockIdx.x * blockDim.x + threadIdx.x; chunk < nchunks;
+       chunk += gridDim.x * blockDim.x) {
+    const uint32_t beg = chunk * (uint32_t)S2;
+    const uint32_t end = min(n_in, beg + (uint32_t)S2);
+    const uint32_t prev_key = beg ? (in_keys[beg - 1] & ~KEY_REAL) : KEY_NONE;
+    const uint32_t next_key = end < n_in ? (in_keys[end] & ~KEY_REAL) : KEY_NONE;
+    const uint32_t first_key = in_keys[beg] & ~KEY_REAL;
+    const uint32_t last_key = in_keys[end - 1] & ~KEY_REAL;
+    bool head_written = false, tail_written = false;
+
+    typename EC_::Xyzz acc;
+    EC_::set_inf(acc);
+    bool any_real = false;
+    uint32_t cur = first_key;
+    bool first_run = true;
+    auto flush = [&](bool last_run) {
+      if (!any_real) return;
+      const bool open_l = first_run && prev_key == cur;
+      const bool open_r = last_run && next_key == cur;
+      if (!open_l && !open_r) {
+        EC_::store(buckets + (size_t)cur * 4 * N, acc);
+      } else {
+        const uint32_t s = open_l ? 2 * chunk : 2 * chunk + 1;
+        out_keys[s] = cur | KEY_REAL;
+        EC_::store(out_pay + (size_t)s * 4 * N, acc);
+        if (open_l) head_written = true; else tail_written = true;
+      }
+    };
+    for (uint32_t j = beg; j < end; ++j) {
+      const uint32_t kr = in_keys[j];
+      const uint32_t key = kr & ~KEY_REAL;
+      if (key != cur) {
+        flush(false);
+        EC_::set_inf(acc);
+        any_real = false;
+        cur = key;
+        first_run = false;
+      }
+      if (kr & KEY_REAL) {
+        typename EC_::Xyzz b;
+        EC_::load(b, in_pay + (size_t)j * 4 * N);
+        ec_add<C>(acc, b);
+        any_real = true;
+      }
+    }
+    flush(true);
+    if (!head_written) out_keys[2 * chunk] = first_key;
+    if (!tail_written) out_keys[2 * chunk + 1] = last_key;
+  }
+}
+
+// ------------------------------------------------- a6 bucket reduction
+// Thread (t, g) owns buckets j = g*s+1 .. g*s+s of window t (digit j is stored
+// at index j-1).  Running sums from the top give R = sum_u X_u and
+// T = sum_u (u+1) X_u; the segment's share of W_t = sum_j j B_j is
+// T + (g s) R (PAPER.md:239's prefix-sum reduction, segmented).
+template <class C>
+__global__ void __launch_bounds__(128) k_reduce_seg(const uint32_t* __restrict__ buckets,
+                                                    const uint32_t* __restrict__ offsets, int W, uint32_t B,
+                                                    int s, uint32_t* __restrict__ seg_out) {
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  const uint32_t G = B / s;
+  const uint32_t total = (uint32_t)W * G;
+  for (uint32_t id = blockIdx.x * blockDim.x + threadIdx.x; id < total; id += gridDim.x * blockDim.x) {
+    const uint32_t t = id / G, g = id % G;
+    typename EC_::Xyzz R, T;
+    EC_::set_inf(R);
+    EC_::set_inf(T);
+    for (int u = s - 1; u >= 0; --u) {
+      const uint32_t key = t * B + g * s + u;
+      if (offsets[key + 1] != offsets[key]) {
+        typename EC_::Xyzz X;
+        EC_::load(X, buckets + (size_t)key * 4 * N);
+        ec_add<C>(R, X);
+      }
+      ec_add<C>(T, R);
+    }
+    ec_mul_small<C>(R, g * (uint32_t)s);
+    ec_add<C>(T, R);
+    EC_::store(seg_out + (size_t)id * 4 * N, T);
+  }
+}
+
+// one block per window: W_t = sum_g seg_out[t][g]
+template <class C>
+__global__ void __launch_bounds__(128) k_reduce_win(const uint32_t* __restrict__ seg_out, uint32_t G,
+                                                    uint32_t* __restrict__ win_out) {
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  extern __shared__ __align__(16) uint32_t red_smem[];
+  const uint32_t t = blockIdx.x;
+  typename EC_::Xyzz acc;
+  EC_::set_inf(acc);
+  for (uint32_t g = threadIdx.x; g < G; g += blockDim.x) {
+    typename EC_::Xyzz X;
+    EC_::load(X, seg_out + ((size_t)t * G + g) * 4 * N);
+    ec_add<C>(acc, X);
+  }
+  EC_::store(red_smem + threadIdx.x * 4 * N, acc);
+  __syncthreads();
+  for (uint32_t w = blockDim.x / 2; w > 0; w >>= 1) {
+    if (threadIdx.x < w) {
+      typename EC_::Xyzz X;
+      EC_::load(X, red_smem + (threadIdx.x + w) * 4 * N);
+      ec_add<C>(acc, X);
+      EC_::store(red_smem + threadIdx.x * 4 * N, acc);
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) EC_::store(win_out + (size_t)t * 4 * N, acc);
+}
+
+// ----------------------------------------- a7 window combination + a8 output
+// Q = sum_t 2^(ct) W_t by Horner from the top window.  out_partial (XYZZ) and/or
+// out_affine (canonical) may be null.
+template <class C>
+__global__ void k_tail(const uint32_t* __restrict__ win_out, int W, int c, uint32_t* __restrict__ out_partial,
+                       uint32_t* __restrict__ out_affine) {
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  if (threadIdx.x || blockIdx.x) return;
+  typename EC_::Xyzz Q;
+  EC_::load(Q, win_out + (size_t)(W - 1) * 4 * N);
+  for (int t = W - 2; t >= 0; --t) {
+    for (int k = 0; k < c; ++k) ec_dbl<C>(Q);
+    typename EC_::Xyzz X;
+    EC_::load(X, win_out + (size_t)t * 4 * N);
+    ec_add<C>(Q, X);
+  }
+  if (EC_::is_inf(Q)) EC_::set_inf(Q);
+  if (out_partial) EC_::store(out_partial, Q);
+  if (out_affine) {
+    uint32_t x[N], y[N];
+    ec_to_affine<C>(x, y, Q);
+    EC_::st(out_affine, x);
+    EC_::st(out_affine + N, y);
+  }
+}
+
+// sum of `count` XYZZ partials in index order, normalised
+template <class C>
+__global__ void k_combine(const uint32_t* __restrict__ partials, int count, uint32_t* __restrict__ out_affine) {
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  if (threadIdx.x || blockIdx.x) return;
+  typename EC_::Xyzz Q;
+  EC_::set_inf(Q);
+  for (int g = 0; g < count; ++g) {
+    typename EC_::Xyzz X;
+    EC_::load(X, partials + (size_t)g * 4 * N);
+    ec_add<C>(Q, X);
+  }
+  uint32_t x[N], y[N];
+  ec_to_affine<C>(x, y, Q);
+  EC_::st(out_affine, x);
+  EC_::st(out_affine + N, y);
+}
+
+// ---------------------------------------- fixed-base generator (bench inputs)
+template <class C>
+__global__ void __launch_bounds__(128) k_fixed_base(const uint32_t* __restrict__ sc, size_t n,
+                                                    uint32_t* __restrict__ out) {
+  using Fp = F<C>;
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  uint32_t gx[N], gy[N];
+#pragma unroll
+  for (int i = 0; i < N; ++i) { gx[i] = C::GX(i); gy[i] = C::GY(i); }
+  Fp::to_mont(gx, gx);
+  Fp::to_mont(gy, gy);
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    const uint32_t* k = sc + i * C::NS;
+    typename EC_::Xyzz Q;
+    bool inf = true;
+    for (int b = C::NS * 32 - 1; b >= 0; --b) {
+      if (!inf) { ec_dbl<C>(Q); inf = EC_::is_inf(Q); }
+      if ((__ldg(k + (b >> 5)) >> (b & 31)) & 1u) {
+        if (inf) { EC_::from_affine(Q, gx, gy); inf = false; }
+        else { ec_madd<C>(Q, gx, gy); inf = EC_::is_inf(Q); }
+      }
+    }
+    if (inf) EC_::set_inf(Q);
+    uint32_t x[N], y[N];
+    ec_to_affine<C>(x, y, Q);
+    EC_::st(out + i * 2 * N, x);
+    EC_::st(out + i * 2 * N + N, y);
+  }
+}
+
+// ------------------------------------------------- diagnostics (tests only)
+template <class C>
+__global__ void k_field_op(int op, const uint32_t* __restrict__ a, const uint32_t* __restrict__ b,
+                           uint32_t* __restrict__ out, size_t n) {
+  using Fp = F<C>;
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    uint32_t x[N], y[N], r[N];
+    EC_::ld(x, a + i * N);
+    EC_::ld(y, b + i * N);
+    switch (op) {
+      case 0: Fp::to_mont(x, x); Fp::to_mont(y, y); Fp::mul(r, x, y); Fp::from_mont(r, r); break;
+      case 1: Fp::add(r, x, y); break;
+      case 2: Fp::sub(r, x, y); break;
+      case 3: Fp::inv_canonical(r, x); break;
+      default: Fp::to_mont(r, x); Fp::from_mont(r, r); break;
+    }
+    EC_::st(out + i * N, r);
+  }
+}
+
+template <class C>
+__global__ void k_ec_op(int op, const uint32_t* __restrict__ P, const uint32_t* __restrict__ Q,
+                        uint32_t* __restrict__ out, size_t n) {
+  using Fp = F<C>;
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    uint32_t px[N], py[N], qx[N], qy[N];
+    EC_::ld(px, P + i * 2 * N); EC_::ld(py, P + i * 2 * N + N);
+    EC_::ld(qx, Q + i * 2 * N); EC_::ld(qy, Q + i * 2 * N + N);
+    const bool p_inf = Fp::is_zero(px) && Fp::is_zero(py);
+    const bool q_inf = Fp::is_zero(qx) && Fp::is_zero(qy);
+    Fp::to_mont(px, px); Fp::to_mont(py, py); Fp::to_mont(qx, qx); Fp::to_mont(qy, qy);
+    typename EC_::Xyzz A, B;
+    if (p_inf) EC_::set_inf(A); else EC_::from_affine(A, px, py);
+    if (q_inf) EC_::set_inf(B); else EC_::from_affine(B, qx, qy);
+    // make A a genuinely projective point (ZZ != 1) by doubling twice and
+    // halving back is not possible; instead scale: (X l^2, Y l^3, ZZ l^2, ZZZ l^3)
+    if (!p_inf) {
+      uint32_t l[N], l2[N], l3[N];
+      Fp::add(l, py, px); Fp::add(l, l, px);           // some nonzero-ish lambda
+      if (Fp::is_zero(l)) Fp::set_one(l);
+      Fp::sqr(l2, l); Fp::mul(l3, l2, l);
+      Fp::mul(A.X, A.X, l2); Fp::mul(A.ZZ, A.ZZ, l2);
+      Fp::mul(A.Y, A.Y, l3); Fp::mul(A.ZZZ, A.ZZZ, l3);
+    }
+    switch (op) {
+      case 0:
+        if (q_inf) break;
+        if (p_inf) EC_::from_affine(A, qx, qy); else ec_madd<C>(A, qx, qy);
+        break;
+      case 1: ec_add<C>(A, B); break;
+      case 2: ec_dbl<C>(A); break;
+      default:
+        if (p_inf) EC_::set_inf(A); else ec_mdbl<C>(A, px, py);
+        break;
+    }
+    uint32_t x[N], y[N];
+    ec_to_affine<C>(x, y, A);
+    EC_::st(out + i * 2 * N, x);
+    EC_::st(out + i * 2 * N + N, y);
+  }
+}
+
+}  // namespace gzkp

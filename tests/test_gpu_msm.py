@@ -1,0 +1,178 @@
+"""GPU MSM parity (`-m gpu`): libgzkp.so through the C ABI vs the oracle,
+bit-exact (the MSM value is unique and the affine encoding canonical, so there
+is no tolerance: DESIGN.md §Parity).
+
+Small n: the C oracle on the full input (same seeded points/scalars).
+Edge cases: n = 0, 1, ragged n, identity points, duplicates, cancellation,
+sparse/adversarial scalar presets, toy curves where buckets constantly hit
+P == Q and P == -Q.
+Invariance: the bytes do not depend on the window size c, the chunk size or
+the sharding (partials + combine)."""
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from oracle import curves, ref
+from tests.fixtures import oracle_msm_cached, oracle_points
+from tests.gpu_util import dev, host, require_cuda
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(autouse=True)
+def _reset_config():
+    yield
+    try:
+        import paper_conf_asplos_maxsm0k0zsh23_b200 as gz
+        gz.set_config(0, 0)
+    except Exception:
+        pass
+
+
+def run(gz, curve, pts, k):
+    return host(gz.msm(curve, dev(pts), dev(k)))
+
+
+def test_config1_bn254_2p10_bit_exact():
+    """BASELINE configs[0]: BN254 n = 2^10, uniform scalars, full oracle check."""
+    gz = require_cuda()
+    pts, _ = oracle_points("bn254", 1 << 10)
+    k = synth.scalars("bn254", 1 << 10, synth.scalar_seed(1))
+    want = oracle_msm_cached("bn254", pts, k)
+    assert np.array_equal(run(gz, "bn254", pts, k), want)
+
+
+@pytest.mark.parametrize("curve,n", [
+    ("bn254", 1), ("bn254", 2), ("bn254", 3), ("bn254", 31), ("bn254", 257), ("bn254", 1000),
+    ("bls12_381", 1), ("bls12_381", 5), ("bls12_381", 257), ("bls12_381", 1024),
+    ("mnt4_753", 1), ("mnt4_753", 7), ("mnt4_753", 64),
+    ("toy_a0", 1), ("toy_a0", 100), ("toy_a0", 3000),
+    ("toy_a2", 1), ("toy_a2", 100), ("toy_a2", 3000),
+])
+def test_msm_uniform_vs_oracle(curve, n):
+    gz = require_cuda()
+    m = max(n, 64) if curve != "mnt4_753" else 64
+    pts, _ = oracle_points(curve, m)
+    pts = pts[:n]
+    k = synth.scalars(curve, n, 500 + n)
+    assert np.array_equal(run(gz, curve, pts, k), oracle_msm_cached(curve, pts, k))
+
+
+def test_msm_empty():
+    gz = require_cuda()
+    for curve in ("bn254", "bls12_381", "mnt4_753"):
+        L = gz.field_limbs(curve)
+        out = run(gz, curve, np.zeros((0, 2 * L), np.uint32), np.zeros((0, gz.scalar_limbs(curve)), np.uint32))
+        assert not out.any()
+
+
+@pytest.mark.parametrize("dist", ["zcash_like", "all_one", "r_minus_1", "single_hot", "pow2", "small",
+                                  "full_bits", "all_zero"])
+@pytest.mark.parametrize("curve", ["bn254", "bls12_381"])
+def test_msm_distributions(curve, dist):
+    gz = require_cuda()
+    n = 700
+    pts, _ = oracle_points(curve, 1024)
+    pts = pts[:n]
+    k = synth.scalars(curve, n, 77, dist)
+    assert np.array_equal(run(gz, curve, pts, k), oracle_msm_cached(curve, pts, k))
+
+
+def test_identity_duplicates_cancellation():
+    gz = require_cuda()
+    curve = "bls12_381"
+    c = curves.get(curve)
+    pts, _ = oracle_points(curve, 1024)
+    pts = pts[:300].copy()
+    k = synth.scalars(curve, 300, 5)
+    pts[3] = 0                         # identity inputs
+    pts[4] = 0
+    pts[10:40] = pts[9]                # duplicated point in many buckets
+    pts[50] = pts[51]                  # P and -P with equal scalars -> cancel
+    y = ref.limbs_to_int(pts[51, c.limbs:])
+    pts[50, c.limbs:] = ref.int_to_limbs((-y) % c.p, c.limbs)
+    k[50] = k[51]
+    # k_i and r - k_i on the same point: sum is O
+    pts[60] = pts[61]
+    kv = ref.limbs_to_int(k[61])
+    k[60] = ref.int_to_limbs((c.r - kv) % c.r, c.scalar_limbs)
+    assert np.array_equal(run(gz, curve, pts, k), oracle_msm_cached(curve, pts, k))
+
+
+def test_result_identity():
+    gz = require_cuda()
+    curve = "bn254"
+    c = curves.get(curve)
+    pts, _ = oracle_points(curve, 1024)
+    P = np.tile(pts[7], (2, 1))
+    k = np.zeros((2, c.scalar_limbs), np.uint32)
+    k[0] = ref.int_to_limbs(12345, c.scalar_limbs)
+    k[1] = ref.int_to_limbs(c.r - 12345, c.scalar_limbs)
+    assert not run(gz, curve, P, k).any()
+
+
+@pytest.mark.parametrize("curve", ["bn254", "bls12_381", "toy_a2"])
+def test_invariance_window_and_chunk(curve):
+    """Same bytes for every c and chunk size (the group is exact)."""
+    gz = require_cuda()
+    n = 2000
+    pts, _ = oracle_points(curve, 2048)
+    pts = pts[:n]
+    k = synth.scalars(curve, n, 31, "zcash_like" if curve != "toy_a2" else "uniform")
+    want = oracle_msm_cached(curve, pts, k)
+    cmax = 16 if curve != "toy_a2" else 4
+    for c in sorted({2, 3, 4, 7, 10, 13, cmax} & set(range(2, cmax + 1))):
+        for S in (1, 3, 16, 64, 257):
+            gz.set_config(c, S)
+            got = run(gz, curve, pts, k)
+            assert np.array_equal(got, want), (c, S)
+
+
+@pytest.mark.parametrize("curve", ["bn254", "bls12_381"])
+def test_sharding_partials_combine(curve):
+    """gzkp_msm_partial on G shards + gzkp_combine_partials == full MSM, for
+    G = 1..8 (the multi-GPU maths on one GPU)."""
+    gz = require_cuda()
+    n = 1000
+    pts, _ = oracle_points(curve, 1024)
+    pts = pts[:n]
+    k = synth.scalars(curve, n, 8)
+    want = oracle_msm_cached(curve, pts, k)
+    L = gz.field_limbs(curve)
+    for G in range(1, 9):
+        parts = []
+        for r in range(G):
+            lo, hi = gz.shard_range(n, G, r)
+            parts.append(gz.msm_partial(curve, dev(pts[lo:hi].reshape(-1, 2 * L)), dev(k[lo:hi].reshape(-1, k.shape[1]))))
+        import torch
+        got = host(gz.combine_partials(curve, torch.stack(parts)))
+        assert np.array_equal(got, want), G
+
+
+def test_prepared_and_host_paths():
+    gz = require_cuda()
+    curve = "bls12_381"
+    pts, _ = oracle_points(curve, 1024)
+    k = synth.scalars(curve, 1024, 12)
+    want = oracle_msm_cached(curve, pts, k)
+    h = gz.PreparedPoints(curve, dev(pts))
+    assert np.array_equal(host(h.msm(dev(k))), want)
+    assert np.array_equal(h.msm_host(k), want)
+    # prefix of a prepared vector
+    want2 = oracle_msm_cached(curve, pts[:100], k[:100])
+    assert np.array_equal(host(h.msm(dev(k[:100]))), want2)
+    h.release()
+    assert np.array_equal(gz.msm_host(curve, pts, k), want)
+
+
+def test_workspace_ex_path():
+    gz = require_cuda()
+    import torch
+    curve = "bn254"
+    pts, _ = oracle_points(curve, 1024)
+    k = synth.scalars(curve, 1024, 13)
+    ws = torch.empty(gz.workspace_bytes(curve, 1024), dtype=torch.uint8, device="cuda")
+    got = host(gz.msm(curve, dev(pts), dev(k), workspace=ws))
+    assert np.array_equal(got, oracle_msm_cached(curve, pts, k))
