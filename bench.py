@@ -200,6 +200,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--window-bits", type=int, default=0)
     ap.add_argument("--chunk", type=int, default=0)
+    ap.add_argument("--workspace", action="store_true", help="caller-provided workspace (gzkp_msm_ex)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     wl = args.workload
@@ -240,9 +241,13 @@ def main():
     comm = gz.Comm(world, rank) if world > 1 else None
     stream = torch.cuda.current_stream()
 
+    ws = None
+    if args.workspace and comm is None:
+        ws = torch.empty(gz.workspace_bytes(curve, n_loc), dtype=torch.uint8, device="cuda")
+
     def step():
         if comm is None:
-            gz.msm(curve, P, K, out=out)
+            gz.msm(curve, P, K, out=out, workspace=ws)
         else:
             gz.msm_sharded(curve, P, K, comm, out=out)
 

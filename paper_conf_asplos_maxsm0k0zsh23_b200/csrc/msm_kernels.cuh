@@ -514,12 +514,14 @@ __global__ void __launch_bounds__(128) k_fixed_base(const uint32_t* __restrict__
   using Fp = F<C>;
   using EC_ = EC<C>;
   constexpr int N = C::N;
-  uint32_t gx[N], gy[N];
-#pragma unroll
-  for (int i = 0; i < N; ++i) { gx[i] = C::GX(i); gy[i] = C::GY(i); }
-  Fp::to_mont(gx, gx);
-  Fp::to_mont(gy, gy);
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    // G in Montgomery form, rebuilt per point (2 muls; keeping it live across
+    // the grid-stride loop miscompiled for the out-of-line N = 24 product)
+    uint32_t gx[N], gy[N];
+#pragma unroll
+    for (int q = 0; q < N; ++q) { gx[q] = C::GX(q); gy[q] = C::GY(q); }
+    Fp::to_mont(gx, gx);
+    Fp::to_mont(gy, gy);
     const uint32_t* k = sc + i * C::NS;
     typename EC_::Xyzz Q;
     bool inf = true;
