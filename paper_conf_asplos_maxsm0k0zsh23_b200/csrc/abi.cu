@@ -10,6 +10,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <map>
 #include <mutex>
 #include <string>
 #include <vector>
@@ -108,6 +109,31 @@ static void init_pool_once() {
 }
 
 static bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
+
+gzkp_status stream_workspace(cudaStream_t s, size_t bytes, void** ptr) {
+  struct Entry { void* p; size_t bytes; };
+  static std::mutex mu;
+  static std::map<std::pair<int, cudaStream_t>, Entry> cache;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lock(mu);
+  Entry& e = cache[{dev, s}];
+  if (e.bytes < bytes) {
+    // stream-ordered: the old buffer is released after the work already queued on s
+    if (e.p) cudaFreeAsync(e.p, s);
+    e.p = nullptr;
+    e.bytes = 0;
+    const size_t want = bytes + bytes / 8;   // headroom against small n changes
+    cudaError_t err = cudaMallocAsync(&e.p, want, s);
+    if (err != cudaSuccess) {
+      e.p = nullptr;
+      return cuda_status(err, "cudaMallocAsync(workspace)");
+    }
+    e.bytes = want;
+  }
+  *ptr = e.p;
+  return GZKP_SUCCESS;
+}
 
 struct Prepared {
   int curve;

@@ -58,6 +58,9 @@ gzkp_status set_error(gzkp_status st, const std::string& msg);
 gzkp_status cuda_status(cudaError_t e, const char* where);
 int device_sm_count();
 bool profiling_enabled();
+// library-owned workspace, one grow-only buffer per (device, stream): calls on
+// one stream are ordered, so they can share it; different streams never do.
+gzkp_status stream_workspace(cudaStream_t s, size_t bytes, void** ptr);
 // profiling hooks (no synchronisation): events[6] recorded by the caller,
 // entries_dev = device address of the call's entry count (copied async).
 struct ProfileRecord {

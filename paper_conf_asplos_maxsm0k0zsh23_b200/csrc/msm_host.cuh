@@ -2,8 +2,9 @@
 //
 // Planner (window size c, chunk size), workspace layout, and the stream-
 // ordered launch sequence.  Everything is enqueued on the caller's stream; no
-// host synchronisation happens inside gzkp_msm (the merge depth is sized from
-// the worst case so no device->host read of the entry count is needed).
+// host synchronisation happens inside gzkp_msm: every data-dependent size
+// (entry count, heavy buckets) is read by the kernels from device memory and
+// the grids are sized for the worst case.
 #pragma once
 #include <cmath>
 #include <cstdlib>
@@ -23,17 +24,15 @@ namespace gzkp {
 struct Plan {
   int c = 0, W = 0;
   uint32_t B = 0;        // buckets per window = 2^(c-1)
-  int S = 64;            // entries per level-0 chunk
-  int S2 = 32;           // slots per merge chunk
+  uint32_t M = 0;        // W * B bucket keys
+  int S = 64;            // entries per accumulation chunk
   int seg = 16;          // buckets per reduction segment
-  int levels = 0;        // merge levels
+  int heavy_levels = 0;  // depth of the heavy-bucket tree
   size_t n = 0;
-  uint64_t E_max = 0;
-  uint64_t slots_max = 0;
+  uint64_t E_max = 0, chunks_max = 0;
   // workspace byte offsets
-  size_t o_pts = 0, o_counts = 0, o_offsets = 0, o_cursor = 0, o_tiles = 0, o_keys = 0, o_vals = 0,
-         o_info = 0, o_slot_k[2] = {0, 0}, o_slot_p[2] = {0, 0}, o_buckets = 0, o_seg = 0, o_win = 0,
-         o_partial = 0, total = 0;
+  size_t o_pts = 0, o_codes = 0, o_counts = 0, o_offsets = 0, o_cursor = 0, o_tiles = 0, o_vals = 0,
+         o_spay = 0, o_heavy = 0, o_buckets = 0, o_seg = 0, o_win = 0, total = 0;
 };
 
 template <class C>
@@ -72,6 +71,7 @@ struct Impl {
     p.c = window_bits(n);
     p.W = (C::SCALAR_BITS + 1 + p.c - 1) / p.c;
     p.B = 1u << (p.c - 1);
+    p.M = (uint32_t)p.W * p.B;
     int S = tunables().chunk_entries;
     if (S <= 0) {
       if (const char* e = getenv("GZKP_SEGMENT")) S = atoi(e);
@@ -80,35 +80,24 @@ struct Impl {
     p.S = S;
     p.seg = (int)std::min<uint32_t>(16u, p.B);
     p.E_max = (uint64_t)n * p.W;
-    const uint64_t chunks_max = (p.E_max + p.S - 1) / p.S;
-    p.slots_max = 2 * chunks_max;
-    uint64_t slots = p.slots_max;
-    p.levels = 0;
-    while (true) {
-      ++p.levels;                       // this level consumes `slots`
-      if (slots <= (uint64_t)p.S2) break;
-      slots = 2 * ((slots + p.S2 - 1) / p.S2);
-    }
-    const uint64_t M = (uint64_t)p.W * p.B;
+    p.chunks_max = std::max<uint64_t>(1, (p.E_max + p.S - 1) / p.S);
+    p.heavy_levels = 0;
+    for (uint64_t span = 1; span < p.chunks_max; span *= HEAVY_FAN) ++p.heavy_levels;
     const uint32_t G = p.B / p.seg;
     size_t o = 0;
     auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
     p.o_pts = prepared ? 0 : take(n * 2 * N * 4);
-    p.o_counts = take(M * 4);
-    p.o_offsets = take((M + 1) * 4);
-    p.o_cursor = take(M * 4);
+    p.o_codes = take((size_t)p.W * n * 4);
+    p.o_counts = take((size_t)p.M * 4);
+    p.o_offsets = take(((size_t)p.M + 1) * 4);
+    p.o_cursor = take((size_t)p.M * 4);
     p.o_tiles = take(SCAN_TILE * 4);
-    p.o_keys = take(std::max<uint64_t>(p.E_max, 1) * 4);
     p.o_vals = take(std::max<uint64_t>(p.E_max, 1) * 4);
-    p.o_info = take(sizeof(LevelInfo));
-    for (int b = 0; b < 2; ++b) {
-      p.o_slot_k[b] = take(std::max<uint64_t>(p.slots_max, 2) * 4);
-      p.o_slot_p[b] = take(std::max<uint64_t>(p.slots_max, 2) * 4 * N * 4);
-    }
-    p.o_buckets = take(M * 4 * N * 4);
+    p.o_spay = take(2 * p.chunks_max * 4 * N * 4);
+    p.o_heavy = take(16);
+    p.o_buckets = take((size_t)p.M * 4 * N * 4);
     p.o_seg = take((size_t)p.W * G * 4 * N * 4);
     p.o_win = take((size_t)p.W * 4 * N * 4);
-    p.o_partial = take(4 * N * 4);
     p.total = o;
     return p;
   }
@@ -136,71 +125,55 @@ struct Impl {
     cudaStream_t s = call.stream;
     if (n == 0) {
       if (call.out_affine) GZ_CHECK(cudaMemsetAsync(call.out_affine, 0, 2 * N * 4, s));
-      if (call.out_partial) {
-        // XYZZ identity: ZZ = ZZZ = 0 (X, Y irrelevant)
-        GZ_CHECK(cudaMemsetAsync(call.out_partial, 0, 4 * N * 4, s));
-      }
+      if (call.out_partial) GZ_CHECK(cudaMemsetAsync(call.out_partial, 0, 4 * N * 4, s));  // ZZ = ZZZ = 0: O
       return GZKP_SUCCESS;
     }
     if ((uint64_t)n >= (1ull << 31)) return set_error(GZKP_ERROR_INVALID_VALUE, "n >= 2^31 not supported");
     const Plan p = plan(n, call.prepared);
     if (p.E_max >= (1ull << 32) - 1) return set_error(GZKP_ERROR_INVALID_VALUE, "n * windows >= 2^32");
-
     char* ws = (char*)call.workspace;
-    bool own = false;
     if (!ws) {
-      GZ_CHECK(cudaMallocAsync((void**)&ws, p.total, s));
-      own = true;
+      void* cached = nullptr;
+      if (gzkp_status st = stream_workspace(s, p.total, &cached)) return st;
+      ws = (char*)cached;
     } else if (call.workspace_bytes < p.total) {
       return set_error(GZKP_ERROR_INVALID_VALUE, "workspace too small");
     }
-    gzkp_status st = run(call, p, ws);
-    if (own) {
-      cudaError_t e = cudaFreeAsync(ws, s);
-      if (st == GZKP_SUCCESS && e != cudaSuccess) st = cuda_status(e, "cudaFreeAsync");
-    }
-    return st;
+    return run(call, p, ws);
   }
 
   static gzkp_status run(const MsmCall& call, const Plan& p, char* ws) {
     cudaStream_t s = call.stream;
     const size_t n = call.n;
-    const uint64_t M = (uint64_t)p.W * p.B;
     auto U = [&](size_t off) { return (uint32_t*)(ws + off); };
     ProfileRecord* prof = profile_begin(s);
     int launches = 0;
+    const int sms = device_sm_count();
 
     // a1: points -> Montgomery (skipped for prepared handles)
     const uint32_t* pts = (const uint32_t*)call.points;
     if (!call.prepared) {
-      gzkp_status st = to_mont(call.points, U(p.o_pts), n, s);
-      if (st) return st;
+      if (gzkp_status st = to_mont(call.points, U(p.o_pts), n, s)) return st;
       pts = U(p.o_pts);
       ++launches;
     }
-    // a2: histogram
-    const int hist_threads = 512;
-    const size_t hist_smem = (size_t)p.B * 4;
-    GZ_CHECK(cudaFuncSetAttribute(k_hist<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hist_smem));
-    GZ_CHECK(cudaFuncSetAttribute(k_scatter<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hist_smem));
-    int nb = std::max(1, (2 * device_sm_count() + p.W - 1) / p.W);
-    nb = (int)std::min<size_t>(nb, (n + 1023) / 1024);
-    nb = std::max(nb, 1);
-    dim3 hgrid(nb, p.W);
-    GZ_CHECK(cudaMemsetAsync(U(p.o_counts), 0, M * 4, s));
-    k_hist<C><<<hgrid, hist_threads, hist_smem, s>>>((const uint32_t*)call.scalars, n, p.c, p.B, U(p.o_counts));
+    // a2: digits + histogram
+    GZ_CHECK(cudaMemsetAsync(U(p.o_counts), 0, (size_t)p.M * 4, s));
+    GZ_CHECK(cudaMemsetAsync(U(p.o_heavy), 0, 16, s));
+    const uint32_t bpw = (uint32_t)((n + DIGIT_THREADS - 1) / DIGIT_THREADS);
+    k_digits<C><<<bpw, DIGIT_THREADS, 0, s>>>((const uint32_t*)call.scalars, n, p.c, p.W, p.B, U(p.o_codes),
+                                              U(p.o_counts));
     GZ_CHECK(cudaGetLastError());
-    launches += 1 + 3 + 1 + 1;   // hist, scan x3, plan, scatter
-    // scan -> offsets (+ cursor copy), offsets[M] = E
-    const uint32_t ntiles = (uint32_t)((M + SCAN_TILE - 1) / SCAN_TILE);
-    k_scan_tiles<<<ntiles, SCAN_THREADS, 0, s>>>(U(p.o_counts), U(p.o_offsets), (uint32_t)M, U(p.o_tiles));
-    k_scan_top<<<1, SCAN_THREADS, 0, s>>>(U(p.o_tiles), ntiles, U(p.o_offsets) + M);
-    k_scan_add<<<ntiles, SCAN_THREADS, 0, s>>>(U(p.o_offsets), U(p.o_cursor), (uint32_t)M, U(p.o_tiles));
-    k_plan<<<1, 1, 0, s>>>(U(p.o_offsets), (uint32_t)M, p.S, p.S2, p.levels, (LevelInfo*)U(p.o_info));
-    // a3: scatter
-    k_scatter<C><<<hgrid, hist_threads, hist_smem, s>>>((const uint32_t*)call.scalars, n, p.c, p.B, U(p.o_cursor),
-                                                         U(p.o_keys), U(p.o_vals));
+    // exclusive scan -> offsets (+ cursor copy); offsets[M] = E
+    const uint32_t ntiles = (uint32_t)((p.M + SCAN_TILE - 1) / SCAN_TILE);
+    k_scan_tiles<<<ntiles, SCAN_THREADS, 0, s>>>(U(p.o_counts), U(p.o_offsets), p.M, U(p.o_tiles));
+    k_scan_top<<<1, SCAN_THREADS, 0, s>>>(U(p.o_tiles), ntiles, U(p.o_offsets) + p.M);
+    k_scan_add<<<ntiles, SCAN_THREADS, 0, s>>>(U(p.o_offsets), U(p.o_cursor), p.M, U(p.o_tiles));
+    // a3: scatter into bucket order (window-major grid)
+    k_scatter<<<(unsigned)((uint64_t)bpw * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw, p.B, U(p.o_cursor),
+                                                                         U(p.o_vals));
     GZ_CHECK(cudaGetLastError());
+    launches += 5;
     profile_mark(prof, 1, s);
 
     // a4: accumulation
@@ -212,30 +185,28 @@ struct Impl {
         cudaFuncSetAttribute(k_accum<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         grid = occupancy_grid((const void*)k_accum<C>, threads, smem);
       }
-      const uint64_t chunks_max = (p.E_max + p.S - 1) / p.S;
-      const int g = (int)std::min<uint64_t>(grid, (chunks_max + threads - 1) / threads);
-      k_accum<C><<<std::max(g, 1), threads, smem, s>>>(U(p.o_keys), U(p.o_vals), pts, (const LevelInfo*)U(p.o_info),
-                                                       p.S, U(p.o_buckets), U(p.o_slot_k[1]), U(p.o_slot_p[1]));
+      const int g = (int)std::min<uint64_t>(grid, (p.chunks_max + threads - 1) / threads);
+      k_accum<C><<<std::max(g, 1), threads, smem, s>>>(U(p.o_vals), U(p.o_offsets), p.M, pts, p.S, U(p.o_buckets),
+                                                       U(p.o_spay));
       GZ_CHECK(cudaGetLastError());
       ++launches;
     }
     profile_mark(prof, 2, s);
-    // a5: merge levels (ping-pong slot buffers)
+    // a5: merge of chunk-boundary partials (+ heavy-bucket tree)
     {
       const int threads = 128;
-      static int grid = 0;
-      if (!grid) grid = occupancy_grid((const void*)k_merge<C>, threads, 0);
-      uint64_t slots = p.slots_max;
-      for (int l = 1; l <= p.levels; ++l) {
-        const int in = l & 1, out = in ^ 1;
-        const uint64_t chunks = (slots + p.S2 - 1) / p.S2;
-        const int g = (int)std::min<uint64_t>(grid, (chunks + threads - 1) / threads);
-        k_merge<C><<<std::max(g, 1), threads, 0, s>>>(U(p.o_slot_k[in]), U(p.o_slot_p[in]), (const LevelInfo*)U(p.o_info),
-                                                      l, p.S2, U(p.o_buckets), U(p.o_slot_k[out]), U(p.o_slot_p[out]));
+      const int gm = (int)std::min<uint64_t>((p.M + threads - 1) / threads, (uint64_t)sms * 16);
+      k_merge_bucket<C><<<gm, threads, 0, s>>>(U(p.o_offsets), p.M, p.S, U(p.o_spay), U(p.o_buckets), U(p.o_heavy));
+      GZ_CHECK(cudaGetLastError());
+      const int gh = (int)std::min<uint64_t>((p.chunks_max + threads - 1) / threads, (uint64_t)sms * 8);
+      uint32_t stride = 1;
+      for (int l = 0; l < p.heavy_levels; ++l, stride *= HEAVY_FAN) {
+        k_heavy_level<C><<<gh, threads, 0, s>>>(U(p.o_offsets), p.M, p.S, stride, U(p.o_heavy), U(p.o_spay));
         GZ_CHECK(cudaGetLastError());
-        ++launches;
-        slots = 2 * chunks;
       }
+      k_heavy_final<C><<<gm, threads, 0, s>>>(U(p.o_offsets), p.M, p.S, U(p.o_heavy), U(p.o_spay), U(p.o_buckets));
+      GZ_CHECK(cudaGetLastError());
+      launches += 2 + p.heavy_levels;
     }
     profile_mark(prof, 3, s);
     // a6: bucket reduction
@@ -258,7 +229,7 @@ struct Impl {
     k_tail<C><<<1, 1, 0, s>>>(U(p.o_win), p.W, p.c, (uint32_t*)call.out_partial, (uint32_t*)call.out_affine);
     GZ_CHECK(cudaGetLastError());
     ++launches;
-    profile_end(prof, U(p.o_info), launches, p.c, s);   // LevelInfo::E is its first field
+    profile_end(prof, U(p.o_offsets) + p.M, launches, p.c, s);
     return GZKP_SUCCESS;
   }
 

@@ -1,16 +1,17 @@
 // msm_kernels.cuh -- the Pippenger pipeline kernels (one template per curve).
 //
 // Steps:
-//   a1 k_to_mont       canonical affine -> Montgomery affine        ("P ... unchanged")
-//   a2 k_hist          signed c-bit digits -> per-window bucket histogram
-//      k_scan_*        exclusive scan -> bucket offsets
-//   a3 k_scatter       counting-sort scatter of (bucket key, point idx|sign)  (p_index)
-//   a4 k_accum         equal-work chunks of the sorted entries, XYZZ madd hot loop,
-//                      points staged in shared memory by cp.async
-//   a5 k_merge         level-wise segmented reduction of chunk-boundary partials
-//   a6 k_reduce_seg/_win  bucket reduction sum_j j*B_j by running sums
-//   a7 k_tail          window combination sum_t 2^(ct) W_t (Horner)
-//   a8 k_tail/k_combine   normalise XYZZ -> canonical affine
+//   a1 k_to_mont        canonical affine -> Montgomery affine           ("P ... unchanged")
+//   a2 k_digits         signed c-bit digits of every (point, window) + bucket histogram
+//      k_scan_*         exclusive scan -> bucket offsets (the p_index layout)
+//   a3 k_scatter        counting-sort scatter of (point idx | sign) into bucket order
+//   a4 k_accum          equal-work chunks of the sorted entries, XYZZ madd hot loop, points
+//                       staged in shared memory by cp.async
+//   a5 k_merge_bucket   sum of each bucket's chunk-boundary partials; k_heavy_* for skewed
+//                       buckets (log-depth tree)
+//   a6 k_reduce_seg/_win   bucket reduction sum_j j*B_j by running sums
+//   a7 k_tail           window combination sum_t 2^(ct) W_t (Horner)
+//   a8 k_tail/k_combine normalise XYZZ -> canonical affine
 #pragma once
 #include <cuda_runtime.h>
 
@@ -18,36 +19,32 @@
 
 namespace gzkp {
 
-constexpr uint32_t KEY_REAL = 0x80000000u;   // slot key flag: payload present
-constexpr uint32_t VAL_NEG = 0x80000000u;    // entry flag: negative digit
-constexpr uint32_t KEY_NONE = 0xffffffffu;
-
-// Per-level device counters written by k_plan (all derived from E on device).
-struct LevelInfo {
-  uint32_t E;            // total entries (non-zero digits)
-  uint32_t n[40];        // n[0] = chunks at level 0; n[l] (l>=1) = slots input to merge level l
-};
+constexpr uint32_t VAL_NEG = 0x80000000u;    // entry / digit-code flag: negative digit
+constexpr int MERGE_QMAX = 64;               // partials summed serially per bucket
+constexpr int HEAVY_FAN = 8;                 // fan-in of the heavy-bucket tree
 
 // ---------------------------------------------------------------- digits
 // Booth-style signed recoding: d_t = v_t + k_{ct-1} - 2^c * k_{ct+c-1}, with
 // v_t = bits [ct, ct+c) of k.  Each digit depends only on c+1 bits, so windows
 // are independent; d_t in [-2^(c-1), 2^(c-1)] and sum_t d_t 2^(ct) = k when
 // k < 2^(cW-1), i.e. W = ceil((b+1)/c) (reading R7).
-template <int NS>
-GZ_DEV int booth_digit(const uint32_t* __restrict__ k, int t, int c) {
+// `word(w)` returns scalar word w (0 beyond the scalar).
+template <class WordFn>
+GZ_DEV int booth_digit(WordFn word, int t, int c) {
   const int pos = t * c - 1;
   uint32_t x;
   if (pos < 0) {
-    x = (__ldg(k) << 1);
+    x = word(0) << 1;
   } else {
     const int w = pos >> 5, off = pos & 31;
-    const uint32_t lo = w < NS ? __ldg(k + w) : 0u;
-    const uint32_t hi = (w + 1) < NS ? __ldg(k + w + 1) : 0u;
-    x = __funnelshift_r(lo, hi, off);
+    x = __funnelshift_r(word(w), word(w + 1), off);
   }
   x &= (c >= 31) ? 0xffffffffu : ((2u << c) - 1u);
   return (int)(x >> 1) + (int)(x & 1u) - (int)(((x >> c) & 1u) << c);
 }
+
+// digit code: 0 for a zero digit, else |d| | (d < 0) << 31; bucket key = |d| - 1
+GZ_DEV uint32_t digit_code(int d) { return d ? ((uint32_t)abs(d) | (d < 0 ? VAL_NEG : 0u)) : 0u; }
 
 // ------------------------------------------------------------ a1 to_mont
 template <class C>
@@ -66,29 +63,69 @@ __global__ void k_to_mont(const uint32_t* __restrict__ in, uint32_t* __restrict_
   }
 }
 
-// --------------------------------------------------- a2 histogram (smem)
-// grid = (blocks_per_window, W); block (bx, t) counts window t's digits of
-// points [bx*per, ...) in a shared-memory histogram of B bins, then flushes
-// the non-zero bins with one global atomic each.  Skewed inputs (the sparse
-// witness's bucket 1) contend only in shared memory.
+// ----------------------------------------------- a2 digits + histogram
+// One thread per point.  The block stages its scalars in shared memory
+// (coalesced 16-B loads; [word][thread] layout, conflict-free), each thread
+// derives all W digits, writes the digit codes window-major (codes[t*n + i],
+// coalesced) and counts them into the global bucket histogram with
+// warp-aggregated atomics: lanes holding the same bucket (the sparse witness's
+// hot bucket 1) issue ONE atomic (PAPER.md:243-245 skew).
+constexpr int DIGIT_THREADS = 256;
 template <class C>
-__global__ void k_hist(const uint32_t* __restrict__ sc, size_t n, int c, uint32_t B,
-                       uint32_t* __restrict__ counts) {
-  extern __shared__ uint32_t hist[];
-  const int t = blockIdx.y;
-  for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
-  __syncthreads();
-  const size_t per = (n + gridDim.x - 1) / gridDim.x;
-  const size_t beg = blockIdx.x * per, end = min(n, beg + per);
-  for (size_t i = beg + threadIdx.x; i < end; i += blockDim.x) {
-    const int d = booth_digit<C::NS>(sc + i * C::NS, t, c);
-    if (d) atomicAdd(&hist[abs(d) - 1], 1u);
+__global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __restrict__ sc, size_t n, int c, int W,
+                                                          uint32_t B, uint32_t* __restrict__ codes,
+                                                          uint32_t* __restrict__ counts) {
+  constexpr int NS = C::NS;
+  __shared__ uint32_t s_sc[NS * DIGIT_THREADS];
+  const size_t base = (size_t)blockIdx.x * DIGIT_THREADS;
+  const size_t left = n > base ? n - base : 0;
+  const int rows = left < (size_t)DIGIT_THREADS ? (int)left : DIGIT_THREADS;
+  // coalesced staging: the block's scalars are rows*NS contiguous words
+  for (int q = threadIdx.x; q < rows * NS; q += DIGIT_THREADS) {
+    const int r = q / NS, w = q % NS;
+    s_sc[w * DIGIT_THREADS + r] = __ldg(sc + base * NS + q);
   }
   __syncthreads();
-  for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
-    const uint32_t h = hist[b];
-    if (h) atomicAdd(&counts[(size_t)t * B + b], h);
+  const int tid = threadIdx.x;
+  const bool live = tid < rows;
+  const size_t i = base + tid;
+  auto word = [&](int w) -> uint32_t { return w < NS ? s_sc[w * DIGIT_THREADS + tid] : 0u; };
+  const int lane = tid & 31;
+  for (int t = 0; t < W; ++t) {
+    const uint32_t code = live ? digit_code(booth_digit(word, t, c)) : 0u;
+    if (live) codes[(size_t)t * n + i] = code;
+    if (code) {
+      const uint32_t key = (uint32_t)t * B + (code & ~VAL_NEG) - 1u;
+      const unsigned peers = __match_any_sync(__activemask(), key);
+      if (lane == __ffs(peers) - 1) atomicAdd(&counts[key], (uint32_t)__popc(peers));
+    }
   }
+}
+
+// ------------------------------------------------------ a3 scatter (sort)
+// Window-major 1-D grid (block b covers window b / bpw) so the blocks in
+// flight write into one or two windows' 4n-byte ranges, which stay resident in
+// L2 until their sectors are complete.  Positions come from the bucket cursors
+// (offsets copy) with warp-aggregated atomics: one atomic per distinct bucket
+// per warp; the order inside a bucket is irrelevant (exact abelian sum,
+// DESIGN.md reading R11).
+constexpr int SCATTER_THREADS = 256;
+static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32_t* __restrict__ codes, size_t n,
+                                                             uint32_t bpw, uint32_t B, uint32_t* __restrict__ cursor,
+                                                             uint32_t* __restrict__ vals) {
+  const uint32_t t = blockIdx.x / bpw;
+  const size_t i = (size_t)(blockIdx.x % bpw) * SCATTER_THREADS + threadIdx.x;
+  if (i >= n) return;
+  const uint32_t code = codes[(size_t)t * n + i];
+  if (!code) return;
+  const uint32_t key = t * B + (code & ~VAL_NEG) - 1u;
+  const unsigned peers = __match_any_sync(__activemask(), key);
+  const int lane = threadIdx.x & 31;
+  const int leader = __ffs(peers) - 1;
+  uint32_t pos = 0;
+  if (lane == leader) pos = atomicAdd(&cursor[key], (uint32_t)__popc(peers));
+  pos = __shfl_sync(peers, pos, leader) + __popc(peers & ((1u << lane) - 1u));
+  vals[pos] = (uint32_t)i | (code & VAL_NEG);
 }
 
 // ----------------------------------------------------- scan (exclusive)
@@ -174,57 +211,6 @@ static __global__ void k_scan_add(uint32_t* __restrict__ out, uint32_t* __restri
   }
 }
 
-// ------------------------------------------------------------ plan counts
-static __global__ void k_plan(const uint32_t* __restrict__ offsets, uint32_t M, int S, int S2, int levels,
-                       LevelInfo* __restrict__ info) {
-  if (threadIdx.x || blockIdx.x) return;
-  const uint32_t E = offsets[M];
-  info->E = E;
-  uint32_t chunks = (E + S - 1) / S;
-  info->n[0] = chunks;
-  uint32_t slots = 2 * chunks;
-  for (int l = 1; l <= levels && l < 40; ++l) {
-    info->n[l] = slots;
-    slots = 2 * ((slots + S2 - 1) / S2);
-  }
-}
-
-// ------------------------------------------------------- a3 scatter (sort)
-// Same grid as k_hist.  Block-local counts are reserved in the global bucket
-// ranges with one atomic per non-zero bin; entries then take consecutive
-// positions from a shared-memory cursor.
-template <class C>
-__global__ void k_scatter(const uint32_t* __restrict__ sc, size_t n, int c, uint32_t B,
-                          uint32_t* __restrict__ cursor, uint32_t* __restrict__ keys,
-                          uint32_t* __restrict__ vals) {
-  extern __shared__ uint32_t hist[];
-  const int t = blockIdx.y;
-  for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) hist[b] = 0;
-  __syncthreads();
-  const size_t per = (n + gridDim.x - 1) / gridDim.x;
-  const size_t beg = blockIdx.x * per, end = min(n, beg + per);
-  for (size_t i = beg + threadIdx.x; i < end; i += blockDim.x) {
-    const int d = booth_digit<C::NS>(sc + i * C::NS, t, c);
-    if (d) atomicAdd(&hist[abs(d) - 1], 1u);
-  }
-  __syncthreads();
-  for (uint32_t b = threadIdx.x; b < B; b += blockDim.x) {
-    const uint32_t h = hist[b];
-    hist[b] = h ? atomicAdd(&cursor[(size_t)t * B + b], h) : 0u;
-  }
-  __syncthreads();
-  const uint32_t kbase = (uint32_t)t * B;
-  for (size_t i = beg + threadIdx.x; i < end; i += blockDim.x) {
-    const int d = booth_digit<C::NS>(sc + i * C::NS, t, c);
-    if (d) {
-      const uint32_t b = abs(d) - 1;
-      const uint32_t pos = atomicAdd(&hist[b], 1u);
-      keys[pos] = kbase + b;
-      vals[pos] = (uint32_t)i | (d < 0 ? VAL_NEG : 0u);
-    }
-  }
-}
-
 // ---------------------------------------------------------- cp.async glue
 GZ_DEV void cp_async16(void* smem, const void* gmem) {
   const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
@@ -248,18 +234,31 @@ struct Stage {
 };
 
 // -------------------------------------------------- a4 bucket accumulation
-// Persistent grid-stride loop over chunks of S consecutive sorted entries.  A
-// chunk may cut through buckets: runs that lie wholly inside the chunk are
-// written straight to their bucket; a run touching the chunk boundary (its
-// bucket continues in the neighbouring chunk) becomes a "boundary partial" in
-// slot 2*chunk (first run) or 2*chunk+1 (last run) for the merge levels.
-// Unused slots carry the chunk's first / last key as a payload-less dummy so
-// the slot keys stay sorted.
+// Persistent grid-stride loop over chunks of S consecutive sorted entries
+// (equal work per thread whatever the bucket sizes: PAPER.md:247-255's load
+// balancing by construction).  Buckets are recovered from the offsets array
+// (bucket k owns entries [off[k], off[k+1])).  A run of one bucket that lies
+// wholly inside the chunk is written straight to the bucket; a run touching a
+// chunk boundary (its bucket continues next door) becomes a boundary partial:
+// the chunk's first run, continuing from the left, goes to slot 2*chunk, the
+// last run, continuing to the right, to slot 2*chunk+1.  A bucket spanning
+// chunks t0..t1 therefore has its partials at slot 2*t0+1 and the head slots
+// 2*t of t0 < t <= t1 (k_merge_bucket relies on this).
 template <class C>
-__global__ void __launch_bounds__(128) k_accum(const uint32_t* __restrict__ keys, const uint32_t* __restrict__ vals,
-                                               const uint32_t* __restrict__ pts, const LevelInfo* __restrict__ info,
-                                               int S, uint32_t* __restrict__ buckets,
-                                               uint32_t* __restrict__ skeys, uint32_t* __restrict__ spay) {
+GZ_DEV uint32_t find_bucket(const uint32_t* __restrict__ off, uint32_t M, uint32_t pos) {
+  // largest k with off[k] <= pos (off non-decreasing, off[0] = 0, pos < off[M])
+  uint32_t lo = 0, hi = M;   // invariant: off[lo] <= pos < off[hi]
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (__ldg(off + mid) <= pos) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+template <class C>
+__global__ void __launch_bounds__(128) k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off,
+                                               uint32_t M, const uint32_t* __restrict__ pts, int S,
+                                               uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay) {
   using Fp = F<C>;
   using EC_ = EC<C>;
   using St = Stage<C>;
@@ -267,42 +266,30 @@ __global__ void __launch_bounds__(128) k_accum(const uint32_t* __restrict__ keys
   extern __shared__ __align__(16) uint32_t stage_smem[];
   uint32_t* slot = stage_smem + threadIdx.x * St::SLOT_WORDS;
 
-  const uint32_t E = info->E;
-  const uint32_t nchunks = info->n[0];
+  const uint32_t E = __ldg(off + M);
+  const uint32_t nchunks = (E + S - 1) / S;
   for (uint32_t chunk = blockIdx.x * blockDim.x + threadIdx.x; chunk < nchunks;
        chunk += gridDim.x * blockDim.x) {
     const uint32_t beg = chunk * (uint32_t)S;
     const uint32_t end = min(E, beg + (uint32_t)S);
-    const uint32_t prev_key = beg ? keys[beg - 1] : KEY_NONE;
-    const uint32_t next_key = end < E ? keys[end] : KEY_NONE;
-    const uint32_t first_key = keys[beg];
-    const uint32_t last_key = keys[end - 1];
-    bool head_written = false, tail_written = false;
+    uint32_t cur = find_bucket<C>(off, M, beg);
+    uint32_t nxt = __ldg(off + cur + 1);
+    bool first_run = true;
 
     typename EC_::Xyzz acc;
     bool acc_inf = true;
-    uint32_t cur = first_key;
-    bool first_run = true;
-
     auto flush = [&](bool last_run) {
-      const bool open_l = first_run && prev_key == cur;
-      const bool open_r = last_run && next_key == cur;
+      const bool open_l = first_run && __ldg(off + cur) < beg;
+      const bool open_r = last_run && nxt > end;
       if (acc_inf) EC_::set_inf(acc);
-      if (!open_l && !open_r) {
-        EC_::store(buckets + (size_t)cur * 4 * N, acc);
-      } else {
-        const uint32_t s = open_l ? 2 * chunk : 2 * chunk + 1;
-        skeys[s] = cur | KEY_REAL;
-        EC_::store(spay + (size_t)s * 4 * N, acc);
-        if (open_l) head_written = true; else tail_written = true;
-      }
+      if (!open_l && !open_r) EC_::store(buckets + (size_t)cur * 4 * N, acc);
+      else EC_::store(spay + (size_t)(open_l ? 2 * chunk : 2 * chunk + 1) * 4 * N, acc);
     };
 
     uint32_t v_next = vals[beg];
     St::fetch(slot, pts, v_next & ~VAL_NEG);
     cp_async_commit();
     for (uint32_t j = beg; j < end; ++j) {
-      const uint32_t key = keys[j];
       const uint32_t v = v_next;
       const int buf = (j - beg) & 1;
       if (j + 1 < end) {
@@ -311,11 +298,11 @@ __global__ void __launch_bounds__(128) k_accum(const uint32_t* __restrict__ keys
       }
       cp_async_commit();
       cp_async_wait<1>();
-      if (key != cur) {
+      if (j == nxt) {                       // bucket boundary: close the run
         flush(false);
         acc_inf = true;
-        cur = key;
         first_run = false;
+        do { ++cur; nxt = __ldg(off + cur + 1); } while (nxt == j);   // skip empty buckets
       }
       uint32_t x[N], y[N];
       EC_::ld(x, slot + buf * St::PT_WORDS);
@@ -332,70 +319,88 @@ __global__ void __launch_bounds__(128) k_accum(const uint32_t* __restrict__ keys
     }
     cp_async_wait<0>();
     flush(true);
-    if (!head_written) skeys[2 * chunk] = first_key;
-    if (!tail_written) skeys[2 * chunk + 1] = last_key;
   }
 }
 
-// --------------------------------------------------------- a5 merge level
-// Same run logic over slots (key|REAL, XYZZ payload) with the full XYZZ add.
+// ----------------------------------------------------------- a5 merge
+// Thread per bucket: a bucket spanning chunks t0 < t1 has q = t1 - t0 + 1
+// partials (slot 2*t0+1, then head slots 2*t).  q <= MERGE_QMAX: summed here.
+// Larger q (a heavy bucket of a skewed input) raises *heavy and is reduced by
+// the k_heavy_level tree instead.
 template <class C>
-__global__ void __launch_bounds__(128) k_merge(const uint32_t* __restrict__ in_keys, const uint32_t* __restrict__ in_pay,
-                                               const LevelInfo* __restrict__ info, int level, int S2,
-                                               uint32_t* __restrict__ buckets, uint32_t* __restrict__ out_keys,
-                                               uint32_t* __restrict__ out_pay) {
+__global__ void __launch_bounds__(128) k_merge_bucket(const uint32_t* __restrict__ off, uint32_t M, int S,
+                                                      const uint32_t* __restrict__ spay, uint32_t* __restrict__ buckets,
+                                                      uint32_t* __restrict__ heavy) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
-  const uint32_t n_in = info->n[level];
-  const uint32_t nchunks = (n_in + S2 - 1) / S2;
-  for (uint32_t chunk = blockIdx.x * blockDim.x + threadIdx.x; chunk < nchunks;
-       chunk += gridDim.x * blockDim.x) {
-    const uint32_t beg = chunk * (uint32_t)S2;
-    const uint32_t end = min(n_in, beg + (uint32_t)S2);
-    const uint32_t prev_key = beg ? (in_keys[beg - 1] & ~KEY_REAL) : KEY_NONE;
-    const uint32_t next_key = end < n_in ? (in_keys[end] & ~KEY_REAL) : KEY_NONE;
-    const uint32_t first_key = in_keys[beg] & ~KEY_REAL;
-    const uint32_t last_key = in_keys[end - 1] & ~KEY_REAL;
-    bool head_written = false, tail_written = false;
-
-    typename EC_::Xyzz acc;
-    EC_::set_inf(acc);
-    bool any_real = false;
-    uint32_t cur = first_key;
-    bool first_run = true;
-    auto flush = [&](bool last_run) {
-      if (!any_real) return;
-      const bool open_l = first_run && prev_key == cur;
-      const bool open_r = last_run && next_key == cur;
-      if (!open_l && !open_r) {
-        EC_::store(buckets + (size_t)cur * 4 * N, acc);
-      } else {
-        const uint32_t s = open_l ? 2 * chunk : 2 * chunk + 1;
-        out_keys[s] = cur | KEY_REAL;
-        EC_::store(out_pay + (size_t)s * 4 * N, acc);
-        if (open_l) head_written = true; else tail_written = true;
-      }
-    };
-    for (uint32_t j = beg; j < end; ++j) {
-      const uint32_t kr = in_keys[j];
-      const uint32_t key = kr & ~KEY_REAL;
-      if (key != cur) {
-        flush(false);
-        EC_::set_inf(acc);
-        any_real = false;
-        cur = key;
-        first_run = false;
-      }
-      if (kr & KEY_REAL) {
-        typename EC_::Xyzz b;
-        EC_::load(b, in_pay + (size_t)j * 4 * N);
-        ec_add<C>(acc, b);
-        any_real = true;
-      }
+  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < M; k += gridDim.x * blockDim.x) {
+    const uint32_t b0 = __ldg(off + k), b1 = __ldg(off + k + 1);
+    if (b1 == b0) continue;
+    const uint32_t t0 = b0 / S, t1 = (b1 - 1) / S;
+    if (t0 == t1) continue;                              // written by k_accum
+    if (t1 - t0 + 1 > (uint32_t)MERGE_QMAX) { *heavy = 1u; continue; }
+    typename EC_::Xyzz acc, X;
+    EC_::load(acc, spay + (size_t)(2 * t0 + 1) * 4 * N);
+    for (uint32_t t = t0 + 1; t <= t1; ++t) {
+      EC_::load(X, spay + (size_t)(2 * t) * 4 * N);
+      ec_add<C>(acc, X);
     }
-    flush(true);
-    if (!head_written) out_keys[2 * chunk] = first_key;
-    if (!tail_written) out_keys[2 * chunk + 1] = last_key;
+    EC_::store(buckets + (size_t)k * 4 * N, acc);
+  }
+}
+
+// Heavy buckets: in-place tree over their head slots.  Head u (0-based, slot
+// 2*(t0+1+u)) is a level-l leader when u % (stride*FAN) == 0; it absorbs heads
+// u + j*stride, j = 1..FAN-1 (leaders of level l-1).  After ceil(log_FAN q)
+// levels head 0 holds the sum of all heads.
+template <class C>
+__global__ void __launch_bounds__(128) k_heavy_level(const uint32_t* __restrict__ off, uint32_t M, int S,
+                                                     uint32_t stride, const uint32_t* __restrict__ heavy,
+                                                     uint32_t* __restrict__ spay) {
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  if (!*heavy) return;
+  const uint32_t E = __ldg(off + M);
+  const uint32_t nchunks = (E + S - 1) / S;
+  const uint64_t span = (uint64_t)stride * HEAVY_FAN;
+  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < nchunks; t += gridDim.x * blockDim.x) {
+    const uint32_t beg = t * (uint32_t)S;
+    const uint32_t k = find_bucket<C>(off, M, beg);
+    const uint32_t b0 = __ldg(off + k), b1 = __ldg(off + k + 1);
+    if (b0 >= beg) continue;                               // chunk t has no head slot
+    const uint32_t t0 = b0 / S, t1 = (b1 - 1) / S;
+    if (t1 - t0 + 1 <= (uint32_t)MERGE_QMAX) continue;     // light bucket
+    const uint32_t u = t - t0 - 1, nheads = t1 - t0;
+    if (u % span) continue;
+    typename EC_::Xyzz acc, X;
+    EC_::load(acc, spay + (size_t)(2 * t) * 4 * N);
+    for (uint32_t j = 1; j < (uint32_t)HEAVY_FAN; ++j) {
+      const uint64_t v = u + (uint64_t)j * stride;
+      if (v >= nheads) break;
+      EC_::load(X, spay + (size_t)(2 * (t0 + 1 + v)) * 4 * N);
+      ec_add<C>(acc, X);
+    }
+    EC_::store(spay + (size_t)(2 * t) * 4 * N, acc);
+  }
+}
+
+template <class C>
+__global__ void __launch_bounds__(128) k_heavy_final(const uint32_t* __restrict__ off, uint32_t M, int S,
+                                                     const uint32_t* __restrict__ heavy,
+                                                     const uint32_t* __restrict__ spay, uint32_t* __restrict__ buckets) {
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  if (!*heavy) return;
+  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < M; k += gridDim.x * blockDim.x) {
+    const uint32_t b0 = __ldg(off + k), b1 = __ldg(off + k + 1);
+    if (b1 == b0) continue;
+    const uint32_t t0 = b0 / S, t1 = (b1 - 1) / S;
+    if (t1 - t0 + 1 <= (uint32_t)MERGE_QMAX) continue;
+    typename EC_::Xyzz acc, X;
+    EC_::load(acc, spay + (size_t)(2 * t0 + 1) * 4 * N);
+    EC_::load(X, spay + (size_t)(2 * (t0 + 1)) * 4 * N);
+    ec_add<C>(acc, X);
+    EC_::store(buckets + (size_t)k * 4 * N, acc);
   }
 }
 

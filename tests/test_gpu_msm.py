@@ -176,3 +176,27 @@ def test_workspace_ex_path():
     ws = torch.empty(gz.workspace_bytes(curve, 1024), dtype=torch.uint8, device="cuda")
     got = host(gz.msm(curve, dev(pts), dev(k), workspace=ws))
     assert np.array_equal(got, oracle_msm_cached(curve, pts, k))
+
+
+def test_sharded_single_rank_nccl():
+    """gzkp_msm_sharded through a real NCCL communicator (world = 1 on the
+    single-GPU box; the multi-rank maths is covered by the partials test)."""
+    gz = require_cuda()
+    import socket
+
+    import torch.distributed as dist
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", world_size=1, rank=0)
+    try:
+        comm = gz.Comm(1, 0)
+        curve = "bls12_381"
+        pts, _ = oracle_points(curve, 1024)
+        k = synth.scalars(curve, 1024, 21)
+        got = host(gz.msm_sharded(curve, dev(pts), dev(k), comm))
+        assert np.array_equal(got, oracle_msm_cached(curve, pts, k))
+        comm.destroy()
+    finally:
+        dist.destroy_process_group()
