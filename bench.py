@@ -198,6 +198,7 @@ def main():
     ap.add_argument("--workload", default="bls12_381_2p22", choices=sorted(WORKLOADS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-prepared", action="store_true")
     ap.add_argument("--window-bits", type=int, default=0)
     ap.add_argument("--chunk", type=int, default=0)
     ap.add_argument("--workspace", action="store_true", help="caller-provided workspace (gzkp_msm_ex)")
@@ -300,6 +301,41 @@ def main():
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms = float(t.item())
+
+    # ---- the same MSM on prepared weighted points (GZKP cross-window
+    # consolidation): setup-time table, timed like the above
+    prepared = None
+    if world == 1 and not args.no_prepared:
+        t0 = time.perf_counter()
+        hp = gz.PreparedPoints(curve, P, weighted=True)
+        torch.cuda.synchronize()
+        prep_s = time.perf_counter() - t0
+        info = hp.info()
+        for _ in range(args.warmup):
+            hp.msm(K, out=out)
+        torch.cuda.synchronize()
+        gz.set_profiling(True)
+        gz.profile_read(reset=True)
+        pe0, pe1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        pe0.record(stream)
+        for _ in range(args.steps):
+            hp.msm(K, out=out)
+        pe1.record(stream)
+        torch.cuda.synchronize()
+        pprof = gz.profile_read(reset=True)
+        gz.set_profiling(False)
+        p_ms = pe0.elapsed_time(pe1) / args.steps
+        pcalls = max(1, pprof["calls"])
+        p_accum = pprof["phase_ms"]["accumulate"] / pcalls
+        p_ach = pprof["entries"] * madd_imad(L) / (p_accum / 1e3) if p_accum > 0 else 0.0
+        prepared = {"value": n / (p_ms / 1e3), "unit": "points/s", "ms_per_step": p_ms,
+                    "window_bits": info["window_bits"], "windows": info["windows"],
+                    "table_bytes": info["bytes"], "prepare_s": prep_s,
+                    "accum_frac_imad_peak": p_ach / (148 * 64 * float(load_peaks()[0].get("sm_max_mhz", 1965.0)) * 1e6),
+                    "phase_ms_per_step": {k: round(v / pcalls, 4) for k, v in pprof["phase_ms"].items()},
+                    "api": "gzkp_points_prepare (weighted table, setup) + gzkp_msm_prepared (timed)"}
+        hp.release()
+        del hp
     ms_per_step = total_ms / args.steps
     value = n / (ms_per_step / 1e3)
 
@@ -386,7 +422,7 @@ def main():
             "config": {"workload": wl, "curve": curve, "n": n, "scalars": sdist, "baseline_config": desc,
                        "window_bits": int(prof["c"]), "parallelism": f"shard{world}" if world > 1 else "single",
                        "l2": "flushed between steps" if flush_l2 else f"inputs {input_bytes >> 20} MiB/GPU > L2"},
-            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "prepared": prepared,
             "gpu_launches": launches * args.steps,
         }
         print(json.dumps(line), flush=True)

@@ -99,9 +99,23 @@ gzkp_status gzkp_msm_ex(int curve, const void *points_affine, const void *scalar
 gzkp_status gzkp_msm_host(int curve, const void *points_affine_host, const void *scalars_host,
                           size_t n, void *out_host, gzkp_stream stream);
 
-/* --- prepared (device-resident Montgomery) points, PAPER.md:194 ---------- */
+/* --- prepared points, PAPER.md:194 ("P ... remains unchanged for a specific
+ * application", so it is preprocessed once) ------------------------------
+ * weighted = 1: GZKP's cross-window consolidation (§4.1,
+ *   interval M = 1): the library stores the weighted points 2^(c t) P_i for
+ *   every window t (W = ceil((b+1)/c) copies, W*n*2*field_bytes bytes of HBM),
+ *   so all windows accumulate into ONE bucket set and the window reduction
+ *   disappears.  window_bits = 0 lets the planner choose c; later MSMs on the
+ *   handle use that c.
+ * weighted = 0: Montgomery-form copy of the points only (standard pipeline).
+ * gzkp_points_prepare = _ex(window_bits 0, weighted 1), falling back to
+ * weighted 0 if the table does not fit. */
+gzkp_status gzkp_points_prepare_ex(int curve, const void *points_affine, size_t n, int window_bits,
+                                   int weighted, void **handle, gzkp_stream stream);
 gzkp_status gzkp_points_prepare(int curve, const void *points_affine, size_t n, void **handle,
                                 gzkp_stream stream);
+gzkp_status gzkp_prepared_info(const void *handle, int *window_bits, int *windows, int *weighted,
+                               size_t *bytes);
 gzkp_status gzkp_msm_prepared(const void *handle, const void *scalars, size_t n, void *out,
                               gzkp_stream stream);
 /* host-buffer scalars/out with a prepared handle (copies inside, synchronises) */

@@ -53,6 +53,9 @@ def lib():
             "gzkp_msm_ex": ([i32, vp, vp, sz, vp, vp, sz, vp], i32),
             "gzkp_msm_host": ([i32, vp, vp, sz, vp, vp], i32),
             "gzkp_points_prepare": ([i32, vp, sz, ctypes.POINTER(vp), vp], i32),
+            "gzkp_points_prepare_ex": ([i32, vp, sz, i32, i32, ctypes.POINTER(vp), vp], i32),
+            "gzkp_prepared_info": ([vp, ctypes.POINTER(i32), ctypes.POINTER(i32), ctypes.POINTER(i32),
+                                    ctypes.POINTER(sz)], i32),
             "gzkp_msm_prepared": ([vp, vp, sz, vp, vp], i32),
             "gzkp_msm_prepared_host": ([vp, vp, sz, vp, vp], i32),
             "gzkp_points_release": ([vp], i32),
@@ -204,15 +207,28 @@ def msm_host(curve, points: np.ndarray, scalars: np.ndarray, out: Optional[np.nd
 class PreparedPoints:
     """Device-resident Montgomery copy of a fixed point vector."""
 
-    def __init__(self, curve, points, stream=None):
+    def __init__(self, curve, points, stream=None, weighted: Optional[bool] = None, window_bits: int = 0):
+        """weighted=None: library default (weighted-point table when it fits);
+        True/False force GZKP's cross-window consolidation on/off."""
         self.curve = curve_id(curve)
         L = field_limbs(self.curve)
         P = _dev_u32(points, 2 * L, "points")
         self.n = P.shape[0]
         h = ctypes.c_void_p()
-        _check(lib().gzkp_points_prepare(self.curve, P.data_ptr(), self.n, ctypes.byref(h), _stream_ptr(stream)),
-               "gzkp_points_prepare")
+        if weighted is None and window_bits == 0:
+            _check(lib().gzkp_points_prepare(self.curve, P.data_ptr(), self.n, ctypes.byref(h), _stream_ptr(stream)),
+                   "gzkp_points_prepare")
+        else:
+            _check(lib().gzkp_points_prepare_ex(self.curve, P.data_ptr(), self.n, window_bits,
+                                                1 if (weighted is None or weighted) else 0, ctypes.byref(h),
+                                                _stream_ptr(stream)), "gzkp_points_prepare_ex")
         self.handle = h
+
+    def info(self):
+        c, w, wt, b = ctypes.c_int(), ctypes.c_int(), ctypes.c_int(), ctypes.c_size_t()
+        _check(lib().gzkp_prepared_info(self.handle, ctypes.byref(c), ctypes.byref(w), ctypes.byref(wt),
+                                        ctypes.byref(b)), "gzkp_prepared_info")
+        return {"window_bits": c.value, "windows": w.value, "weighted": bool(wt.value), "bytes": b.value}
 
     def msm(self, scalars, out=None, stream=None):
         torch = _torch()
@@ -309,22 +325,27 @@ def ec_op(curve, op: int, P, Q, stream=None):
 
 # ------------------------------------------------------------- multi-GPU
 
+def broadcast_unique_id(rank: int, group=None) -> bytes:
+    """Rank 0 creates the NCCL unique id (gzkp_nccl_unique_id); the default
+    torch process group carries the 128 bytes to every rank (plumbing only)."""
+    torch = _torch()
+    import torch.distributed as dist
+    uid = ctypes.create_string_buffer(128)
+    if rank == 0:
+        _check(lib().gzkp_nccl_unique_id(uid), "gzkp_nccl_unique_id")
+    t = torch.frombuffer(bytearray(uid.raw), dtype=torch.uint8).clone()
+    if dist.get_backend(group) == "nccl":
+        t = t.cuda()
+    dist.broadcast(t, src=0, group=group)
+    return bytes(t.cpu().numpy().tobytes())
+
+
 class Comm:
     """NCCL communicator for gzkp_msm_sharded.  The 128-byte unique id is
     broadcast through the default torch process group (plumbing only)."""
 
     def __init__(self, world: int, rank: int, group=None):
-        torch = _torch()
-        import torch.distributed as dist
-        uid = ctypes.create_string_buffer(128)
-        if rank == 0:
-            _check(lib().gzkp_nccl_unique_id(uid), "gzkp_nccl_unique_id")
-        t = torch.frombuffer(bytearray(uid.raw), dtype=torch.uint8).clone()
-        if dist.get_backend(group) == "nccl":
-            t = t.cuda()
-        dist.broadcast(t, src=0, group=group)
-        raw = bytes(t.cpu().numpy().tobytes())
-        uid = ctypes.create_string_buffer(raw, 128)
+        uid = ctypes.create_string_buffer(broadcast_unique_id(rank, group), 128)
         h = ctypes.c_void_p()
         _check(lib().gzkp_comm_init(world, rank, uid, ctypes.byref(h)), "gzkp_comm_init")
         self.handle = h

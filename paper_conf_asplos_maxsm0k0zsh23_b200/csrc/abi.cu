@@ -138,7 +138,10 @@ gzkp_status stream_workspace(cudaStream_t s, size_t bytes, void** ptr) {
 struct Prepared {
   int curve;
   size_t n;
-  void* pts;   // Montgomery affine, n x 2N u32
+  void* pts;          // Montgomery affine: n x 2N u32, or the W x n weighted-point table
+  bool weighted;      // NEXT-1 table 2^(ct) P_i (cross-window consolidation)
+  int c, W;
+  size_t bytes;
 };
 
 // ------------------------------------------------------------- NCCL (dlopen)
@@ -303,20 +306,54 @@ gzkp_status gzkp_msm_host(int curve, const void* points_host, const void* scalar
   return st;
 }
 
-gzkp_status gzkp_points_prepare(int curve, const void* points_affine, size_t n, void** handle, gzkp_stream stream) {
+gzkp_status gzkp_points_prepare_ex(int curve, const void* points_affine, size_t n, int window_bits, int weighted,
+                                   void** handle, gzkp_stream stream) {
   const CurveImpl* c = impl_for(curve);
   if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
-  if (!handle || (n && !points_affine) || !aligned16(points_affine))
+  if (!handle || (n && !points_affine) || !aligned16(points_affine) || window_bits < 0 || window_bits > 22)
     return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
-  Prepared* h = new (std::nothrow) Prepared{curve, n, nullptr};
+  Prepared* h = new (std::nothrow) Prepared{curve, n, nullptr, false, 0, 1, 0};
   if (!h) return set_error(GZKP_ERROR_OUT_OF_MEMORY, "handle");
-  if (n) {
-    cudaError_t e = cudaMalloc(&h->pts, n * 2 * c->limbs * 4);
+  const size_t pt_bytes = 2 * (size_t)c->limbs * 4;
+  if (weighted == 1 && n) {
+    // weighted-point table 2^(ct) P_i for every window t (M = 1)
+    const int W = c->table_windows(n, window_bits);
+    if ((uint64_t)n * W >= (1ull << 31)) { delete h; return set_error(GZKP_ERROR_INVALID_VALUE, "table >= 2^31 points"); }
+    h->bytes = n * W * pt_bytes;
+    cudaError_t e = cudaMalloc(&h->pts, h->bytes);
+    if (e != cudaSuccess) { delete h; return cuda_status(e, "cudaMalloc(weighted table)"); }
+    gzkp_status st = c->precompute(points_affine, n, window_bits, h->pts, &h->c, &h->W, (cudaStream_t)stream);
+    if (st) { cudaFree(h->pts); delete h; return st; }
+    h->weighted = true;
+  } else if (n) {
+    h->bytes = n * pt_bytes;
+    cudaError_t e = cudaMalloc(&h->pts, h->bytes);
     if (e != cudaSuccess) { delete h; return cuda_status(e, "cudaMalloc(prepared)"); }
     gzkp_status st = c->to_mont(points_affine, h->pts, n, (cudaStream_t)stream);
     if (st) { cudaFree(h->pts); delete h; return st; }
+    h->c = window_bits;
   }
   *handle = h;
+  return GZKP_SUCCESS;
+}
+
+gzkp_status gzkp_points_prepare(int curve, const void* points_affine, size_t n, void** handle, gzkp_stream stream) {
+  // default: the paper's weighted points when they fit, else plain Montgomery points
+  gzkp_status st = gzkp_points_prepare_ex(curve, points_affine, n, 0, 1, handle, stream);
+  if (st == GZKP_ERROR_OUT_OF_MEMORY || st == GZKP_ERROR_INVALID_VALUE) {
+    cudaGetLastError();   // clear a failed allocation
+    st = gzkp_points_prepare_ex(curve, points_affine, n, 0, 0, handle, stream);
+  }
+  return st;
+}
+
+gzkp_status gzkp_prepared_info(const void* handle, int* window_bits, int* windows, int* weighted, size_t* bytes) {
+  const Prepared* h = (const Prepared*)handle;
+  if (!h) return set_error(GZKP_ERROR_INVALID_VALUE, "NULL handle");
+  if (window_bits) *window_bits = h->c;
+  if (windows) *windows = h->W;
+  if (weighted) *weighted = h->weighted ? 1 : 0;
+  if (bytes) *bytes = h->bytes;
   return GZKP_SUCCESS;
 }
 
@@ -330,6 +367,9 @@ gzkp_status gzkp_msm_prepared(const void* handle, const void* scalars, size_t n,
   MsmCall call;
   call.points = h->pts;
   call.prepared = true;
+  call.consolidated = h->weighted;
+  call.window_bits = h->c;
+  call.table_n = h->n;
   call.scalars = scalars;
   call.n = n;
   call.out_affine = out;

@@ -23,6 +23,9 @@ Tunables& tunables();
 struct MsmCall {
   const void* points = nullptr;   // canonical affine, or Montgomery when prepared
   bool prepared = false;
+  bool consolidated = false;      // points = weighted-point table [W][table_n] (NEXT-1)
+  int window_bits = 0;            // forced c (0 = planner); set for consolidated tables
+  size_t table_n = 0;
   const void* scalars = nullptr;
   size_t n = 0;
   void* out_affine = nullptr;     // canonical affine result (may be null)
@@ -45,6 +48,8 @@ struct CurveImpl {
   gzkp_status (*fixed_base)(const void* scalars, size_t n, void* out, cudaStream_t s);
   gzkp_status (*field_op)(int op, const void* a, const void* b, void* out, size_t n, cudaStream_t s);
   gzkp_status (*ec_op)(int op, const void* P, const void* Q, void* out, size_t n, cudaStream_t s);
+  gzkp_status (*precompute)(const void* in, size_t n, int c, void* table, int* c_out, int* w_out, cudaStream_t s);
+  int (*table_windows)(size_t n, int c);
 };
 
 const CurveImpl* impl_bn254();

@@ -24,7 +24,10 @@ namespace gzkp {
 struct Plan {
   int c = 0, W = 0;
   uint32_t B = 0;        // buckets per window = 2^(c-1)
-  uint32_t M = 0;        // W * B bucket keys
+  bool consolidated = false;   // NEXT-1: windows share one bucket set (weighted points)
+  int Wb = 0;            // bucket windows: W, or 1 when consolidated
+  uint32_t val_stride = 0;     // table stride of the weighted points (consolidated)
+  uint32_t M = 0;        // Wb * B bucket keys
   int S = 64;            // entries per accumulation chunk
   int seg = 16;          // buckets per reduction segment
   int heavy_levels = 0;  // depth of the heavy-bucket tree
@@ -32,8 +35,10 @@ struct Plan {
   uint64_t E_max = 0, chunks_max = 0;
   // workspace byte offsets
   size_t o_pts = 0, o_codes = 0, o_counts = 0, o_offsets = 0, o_cursor = 0, o_tiles = 0, o_vals = 0,
-         o_spay = 0, o_heavy = 0, o_buckets = 0, o_seg = 0, o_win = 0, total = 0;
+         o_spay = 0, o_heavy = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_win = 0, total = 0;
 };
+
+constexpr uint32_t WIN_PER_BLOCK = 1024;   // segment partials summed per block (stage A)
 
 template <class C>
 struct Impl {
@@ -65,20 +70,50 @@ struct Impl {
     return best;
   }
 
-  static Plan plan(size_t n, bool prepared) {
+  // Window size when all windows share one bucket set (weighted points): no
+  // window combination, reduction over 2^(c-1) buckets once, so larger c pays.
+  static int window_bits_consolidated(size_t n) {
+    if (const char* e = getenv("GZKP_WINDOW_BITS_PREPARED")) {
+      int v = atoi(e);
+      if (v >= 2 && v <= 22) return v;
+    }
+    const double madd = 10.0, add = 14.0, lat = 6000.0;
+    int best = 8;
+    double best_cost = 1e300;
+    const int cmax = C::SCALAR_BITS < 16 ? 4 : 22;
+    for (int c = 2; c <= cmax; ++c) {
+      const int W = (C::SCALAR_BITS + 1 + c - 1) / c;
+      const double B = std::ldexp(1.0, c - 1);
+      const double entries = (double)n * W * (1.0 - std::ldexp(1.0, -c));
+      const double reduce = B * 3.4 * add + 60.0 * add * lat / 8.0;
+      const double cost = entries * madd + reduce;
+      if (cost < best_cost) { best_cost = cost; best = c; }
+    }
+    return best;
+  }
+
+  static Plan plan(size_t n, bool prepared, bool consolidated = false, int c_forced = 0, size_t table_n = 0) {
     Plan p;
     p.n = n;
-    p.c = window_bits(n);
+    p.consolidated = consolidated;
+    p.c = c_forced > 0 ? c_forced : window_bits(n);
     p.W = (C::SCALAR_BITS + 1 + p.c - 1) / p.c;
     p.B = 1u << (p.c - 1);
-    p.M = (uint32_t)p.W * p.B;
+    p.Wb = consolidated ? 1 : p.W;
+    p.val_stride = consolidated ? (uint32_t)table_n : 0u;
+    p.M = (uint32_t)p.Wb * p.B;
     int S = tunables().chunk_entries;
     if (S <= 0) {
       if (const char* e = getenv("GZKP_SEGMENT")) S = atoi(e);
     }
     if (S <= 0) S = 64;
     p.S = S;
-    p.seg = (int)std::min<uint32_t>(16u, p.B);
+    // reduction segment: up to 16 buckets, fewer when that leaves < ~32K threads
+    {
+      uint64_t seg = 16;
+      while (seg > 1 && (uint64_t)p.Wb * p.B / seg < 32768) seg >>= 1;
+      p.seg = (int)std::min<uint64_t>(seg, p.B);
+    }
     p.E_max = (uint64_t)n * p.W;
     p.chunks_max = std::max<uint64_t>(1, (p.E_max + p.S - 1) / p.S);
     p.heavy_levels = 0;
@@ -96,8 +131,9 @@ struct Impl {
     p.o_spay = take(2 * p.chunks_max * 4 * N * 4);
     p.o_heavy = take(16);
     p.o_buckets = take((size_t)p.M * 4 * N * 4);
-    p.o_seg = take((size_t)p.W * G * 4 * N * 4);
-    p.o_win = take((size_t)p.W * 4 * N * 4);
+    p.o_seg = take((size_t)p.Wb * G * 4 * N * 4);
+    p.o_mid = take((size_t)p.Wb * ((G + WIN_PER_BLOCK - 1) / WIN_PER_BLOCK) * 4 * N * 4);
+    p.o_win = take((size_t)p.Wb * 4 * N * 4);
     p.total = o;
     return p;
   }
@@ -129,8 +165,10 @@ struct Impl {
       return GZKP_SUCCESS;
     }
     if ((uint64_t)n >= (1ull << 31)) return set_error(GZKP_ERROR_INVALID_VALUE, "n >= 2^31 not supported");
-    const Plan p = plan(n, call.prepared);
+    const Plan p = plan(n, call.prepared, call.consolidated, call.window_bits, call.table_n);
     if (p.E_max >= (1ull << 32) - 1) return set_error(GZKP_ERROR_INVALID_VALUE, "n * windows >= 2^32");
+    if (p.consolidated && (uint64_t)p.val_stride * p.W >= (1ull << 31))
+      return set_error(GZKP_ERROR_INVALID_VALUE, "weighted-point table >= 2^31 points");
     char* ws = (char*)call.workspace;
     if (!ws) {
       void* cached = nullptr;
@@ -161,7 +199,8 @@ struct Impl {
     GZ_CHECK(cudaMemsetAsync(U(p.o_counts), 0, (size_t)p.M * 4, s));
     GZ_CHECK(cudaMemsetAsync(U(p.o_heavy), 0, 16, s));
     const uint32_t bpw = (uint32_t)((n + DIGIT_THREADS - 1) / DIGIT_THREADS);
-    k_digits<C><<<bpw, DIGIT_THREADS, 0, s>>>((const uint32_t*)call.scalars, n, p.c, p.W, p.B, U(p.o_codes),
+    const uint32_t key_stride = p.consolidated ? 0u : p.B;
+    k_digits<C><<<bpw, DIGIT_THREADS, 0, s>>>((const uint32_t*)call.scalars, n, p.c, p.W, key_stride, U(p.o_codes),
                                               U(p.o_counts));
     GZ_CHECK(cudaGetLastError());
     // exclusive scan -> offsets (+ cursor copy); offsets[M] = E
@@ -170,8 +209,8 @@ struct Impl {
     k_scan_top<<<1, SCAN_THREADS, 0, s>>>(U(p.o_tiles), ntiles, U(p.o_offsets) + p.M);
     k_scan_add<<<ntiles, SCAN_THREADS, 0, s>>>(U(p.o_offsets), U(p.o_cursor), p.M, U(p.o_tiles));
     // a3: scatter into bucket order (window-major grid)
-    k_scatter<<<(unsigned)((uint64_t)bpw * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw, p.B, U(p.o_cursor),
-                                                                         U(p.o_vals));
+    k_scatter<<<(unsigned)((uint64_t)bpw * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw, key_stride,
+                                                                         p.val_stride, U(p.o_cursor), U(p.o_vals));
     GZ_CHECK(cudaGetLastError());
     launches += 5;
     profile_mark(prof, 1, s);
@@ -213,24 +252,51 @@ struct Impl {
     const uint32_t G = p.B / p.seg;
     {
       const int threads = 128;
-      const uint32_t total = (uint32_t)p.W * G;
-      k_reduce_seg<C><<<(total + threads - 1) / threads, threads, 0, s>>>(U(p.o_buckets), U(p.o_offsets), p.W, p.B,
+      const uint32_t total = (uint32_t)p.Wb * G;
+      k_reduce_seg<C><<<(total + threads - 1) / threads, threads, 0, s>>>(U(p.o_buckets), U(p.o_offsets), p.Wb, p.B,
                                                                           p.seg, U(p.o_seg));
       GZ_CHECK(cudaGetLastError());
       const int rthreads = 128;
       const size_t smem = (size_t)rthreads * 4 * N * 4;
       GZ_CHECK(cudaFuncSetAttribute(k_reduce_win<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      k_reduce_win<C><<<p.W, rthreads, smem, s>>>(U(p.o_seg), G, U(p.o_win));
+      const uint32_t nb = (G + WIN_PER_BLOCK - 1) / WIN_PER_BLOCK;
+      k_reduce_win<C><<<dim3(nb, p.Wb), rthreads, smem, s>>>(U(p.o_seg), G, WIN_PER_BLOCK, U(p.o_mid));
       GZ_CHECK(cudaGetLastError());
-      launches += 2;
+      k_reduce_win<C><<<dim3(1, p.Wb), rthreads, smem, s>>>(U(p.o_mid), nb, nb, U(p.o_win));
+      GZ_CHECK(cudaGetLastError());
+      launches += 3;
     }
     profile_mark(prof, 4, s);
     // a7 + a8
-    k_tail<C><<<1, 1, 0, s>>>(U(p.o_win), p.W, p.c, (uint32_t*)call.out_partial, (uint32_t*)call.out_affine);
+    k_tail<C><<<1, 1, 0, s>>>(U(p.o_win), p.Wb, p.c, (uint32_t*)call.out_partial, (uint32_t*)call.out_affine);
     GZ_CHECK(cudaGetLastError());
     ++launches;
     profile_end(prof, U(p.o_offsets) + p.M, launches, p.c, s);
     return GZKP_SUCCESS;
+  }
+
+  // NEXT-1 prepare: table[t*n + i] = 2^(ct) P_i (Montgomery affine), t < W.
+  // Returns the window bits used (the MSM calls on this table must use them).
+  static gzkp_status precompute(const void* in, size_t n, int c, void* table, int* c_out, int* w_out, cudaStream_t s) {
+    if (c <= 0) c = window_bits_consolidated(n);
+    const int W = (C::SCALAR_BITS + 1 + c - 1) / c;
+    *c_out = c;
+    *w_out = W;
+    if (!n) return GZKP_SUCCESS;
+    uint32_t* T = (uint32_t*)table;
+    if (gzkp_status st = to_mont(in, T, n, s)) return st;
+    const int threads = 128;
+    const int grid = (int)std::min<size_t>((n + threads - 1) / threads, (size_t)device_sm_count() * 32);
+    for (int t = 1; t < W; ++t) {
+      k_precompute_step<C><<<grid, threads, 0, s>>>(T + (size_t)(t - 1) * n * 2 * N, T + (size_t)t * n * 2 * N, n, c);
+      GZ_CHECK(cudaGetLastError());
+    }
+    return GZKP_SUCCESS;
+  }
+
+  static int table_windows(size_t n, int c) {
+    if (c <= 0) c = window_bits_consolidated(n);
+    return (C::SCALAR_BITS + 1 + c - 1) / c;
   }
 
   static gzkp_status combine(const void* partials, int count, void* out, cudaStream_t s) {
@@ -269,7 +335,8 @@ struct Impl {
   static const CurveImpl* get() {
     static const CurveImpl impl = {C::ID, C::N, C::NS, C::SCALAR_BITS,
                                    &Impl::window_bits, &Impl::workspace_bytes, &Impl::msm, &Impl::to_mont,
-                                   &Impl::combine, &Impl::fixed_base, &Impl::field_op, &Impl::ec_op};
+                                   &Impl::combine, &Impl::fixed_base, &Impl::field_op, &Impl::ec_op,
+                                   &Impl::precompute, &Impl::table_windows};
     return &impl;
   }
 };

@@ -73,7 +73,7 @@ __global__ void k_to_mont(const uint32_t* __restrict__ in, uint32_t* __restrict_
 constexpr int DIGIT_THREADS = 256;
 template <class C>
 __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __restrict__ sc, size_t n, int c, int W,
-                                                          uint32_t B, uint32_t* __restrict__ codes,
+                                                          uint32_t key_stride, uint32_t* __restrict__ codes,
                                                           uint32_t* __restrict__ counts) {
   constexpr int NS = C::NS;
   __shared__ uint32_t s_sc[NS * DIGIT_THREADS];
@@ -95,13 +95,17 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
     const uint32_t code = live ? digit_code(booth_digit(word, t, c)) : 0u;
     if (live) codes[(size_t)t * n + i] = code;
     if (code) {
-      const uint32_t key = (uint32_t)t * B + (code & ~VAL_NEG) - 1u;
+      const uint32_t key = (uint32_t)t * key_stride + (code & ~VAL_NEG) - 1u;
       const unsigned peers = __match_any_sync(__activemask(), key);
       if (lane == __ffs(peers) - 1) atomicAdd(&counts[key], (uint32_t)__popc(peers));
     }
   }
 }
 
+// Cross-window consolidation (§4.1; NEXT-1): with prepared
+// weighted points P_{i,t} = 2^(ct) P_i stored as table[t*n + i], every window
+// uses the SAME bucket set: key_stride = 0 and the entry value indexes the
+// table (val_stride = n).  Without it key_stride = B, val_stride = 0.
 // ------------------------------------------------------ a3 scatter (sort)
 // Window-major 1-D grid (block b covers window b / bpw) so the blocks in
 // flight write into one or two windows' 4n-byte ranges, which stay resident in
@@ -111,21 +115,21 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
 // DESIGN.md reading R11).
 constexpr int SCATTER_THREADS = 256;
 static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32_t* __restrict__ codes, size_t n,
-                                                             uint32_t bpw, uint32_t B, uint32_t* __restrict__ cursor,
-                                                             uint32_t* __restrict__ vals) {
+                                                             uint32_t bpw, uint32_t key_stride, uint32_t val_stride,
+                                                             uint32_t* __restrict__ cursor, uint32_t* __restrict__ vals) {
   const uint32_t t = blockIdx.x / bpw;
   const size_t i = (size_t)(blockIdx.x % bpw) * SCATTER_THREADS + threadIdx.x;
   if (i >= n) return;
   const uint32_t code = codes[(size_t)t * n + i];
   if (!code) return;
-  const uint32_t key = t * B + (code & ~VAL_NEG) - 1u;
+  const uint32_t key = t * key_stride + (code & ~VAL_NEG) - 1u;
   const unsigned peers = __match_any_sync(__activemask(), key);
   const int lane = threadIdx.x & 31;
   const int leader = __ffs(peers) - 1;
   uint32_t pos = 0;
   if (lane == leader) pos = atomicAdd(&cursor[key], (uint32_t)__popc(peers));
   pos = __shfl_sync(peers, pos, leader) + __popc(peers & ((1u << lane) - 1u));
-  vals[pos] = (uint32_t)i | (code & VAL_NEG);
+  vals[pos] = (t * val_stride + (uint32_t)i) | (code & VAL_NEG);
 }
 
 // ----------------------------------------------------- scan (exclusive)
@@ -437,17 +441,22 @@ __global__ void __launch_bounds__(128) k_reduce_seg(const uint32_t* __restrict__
   }
 }
 
-// one block per window: W_t = sum_g seg_out[t][g]
+// Group sums: group t holds G consecutive XYZZ points; block (b, t) sums the
+// slice [b*per_block, (b+1)*per_block) of group t into out[t*gridDim.x + b].
+// Launched twice (many blocks per window, then one block per window) so the
+// single-window case (weighted points, 2^19 buckets) is not one block's job.
 template <class C>
 __global__ void __launch_bounds__(128) k_reduce_win(const uint32_t* __restrict__ seg_out, uint32_t G,
-                                                    uint32_t* __restrict__ win_out) {
+                                                    uint32_t per_block, uint32_t* __restrict__ win_out) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
   extern __shared__ __align__(16) uint32_t red_smem[];
-  const uint32_t t = blockIdx.x;
+  const uint32_t t = blockIdx.y;
+  const uint32_t lo = blockIdx.x * per_block;
+  const uint32_t hi = min(G, lo + per_block);
   typename EC_::Xyzz acc;
   EC_::set_inf(acc);
-  for (uint32_t g = threadIdx.x; g < G; g += blockDim.x) {
+  for (uint32_t g = lo + threadIdx.x; g < hi; g += blockDim.x) {
     typename EC_::Xyzz X;
     EC_::load(X, seg_out + ((size_t)t * G + g) * 4 * N);
     ec_add<C>(acc, X);
@@ -463,7 +472,7 @@ __global__ void __launch_bounds__(128) k_reduce_win(const uint32_t* __restrict__
     }
     __syncthreads();
   }
-  if (threadIdx.x == 0) EC_::store(win_out + (size_t)t * 4 * N, acc);
+  if (threadIdx.x == 0) EC_::store(win_out + ((size_t)t * gridDim.x + blockIdx.x) * 4 * N, acc);
 }
 
 // ----------------------------------------- a7 window combination + a8 output
@@ -510,6 +519,39 @@ __global__ void k_combine(const uint32_t* __restrict__ partials, int count, uint
   ec_to_affine<C>(x, y, Q);
   EC_::st(out_affine, x);
   EC_::st(out_affine + N, y);
+}
+
+// ------------------------------------ NEXT-1: weighted-point precompute
+// table[t] = 2^c * table[t-1] (affine Montgomery), one thread per point: c
+// doublings in XYZZ, then one inversion to return to affine.  Run once per
+// point set at prepare time (the proving key is fixed).
+template <class C>
+__global__ void __launch_bounds__(128) k_precompute_step(const uint32_t* __restrict__ prev, uint32_t* __restrict__ next,
+                                                         size_t n, int c) {
+  using Fp = F<C>;
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    uint32_t x[N], y[N];
+    EC_::ld(x, prev + i * 2 * N);
+    EC_::ld(y, prev + i * 2 * N + N);
+    if (Fp::is_zero(x) && Fp::is_zero(y)) {           // O stays O
+      EC_::st(next + i * 2 * N, x);
+      EC_::st(next + i * 2 * N + N, y);
+      continue;
+    }
+    typename EC_::Xyzz Q;
+    EC_::from_affine(Q, x, y);
+    for (int k = 0; k < c; ++k) ec_dbl<C>(Q);
+    uint32_t ax[N], ay[N];
+    ec_to_affine<C>(ax, ay, Q);                         // canonical, O -> (0,0)
+    if (!(Fp::is_zero(ax) && Fp::is_zero(ay))) {
+      Fp::to_mont(ax, ax);
+      Fp::to_mont(ay, ay);
+    }
+    EC_::st(next + i * 2 * N, ax);
+    EC_::st(next + i * 2 * N + N, ay);
+  }
 }
 
 // ---------------------------------------- fixed-base generator (bench inputs)

@@ -42,3 +42,7 @@ def test_closed_form_full_size(curve, log_n, cfg, dist):
     got = host(gz.msm(curve, pts, dev(k)))
     want = oracle.closed_form(curve, k, d)
     assert np.array_equal(got, want)
+    # the same MSM through prepared weighted points (NEXT-1), planner's c
+    h = gz.PreparedPoints(curve, pts, weighted=True)
+    assert np.array_equal(host(h.msm(dev(k))), want)
+    h.release()

@@ -200,3 +200,41 @@ def test_sharded_single_rank_nccl():
         comm.destroy()
     finally:
         dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("curve,cs", [("bn254", (3, 8, 13, 16, 20)), ("bls12_381", (4, 11, 16, 18, 21)),
+                                      ("mnt4_753", (9, 16)), ("toy_a0", (2, 3, 4)), ("toy_a2", (2, 4))])
+def test_weighted_points_cross_window_consolidation(curve, cs):
+    """NEXT-1: prepared weighted points 2^(ct) P_i, one bucket
+    set for all windows; bit-exact vs the oracle for several c, sparse scalars,
+    identity points and a prefix of the prepared vector."""
+    gz = require_cuda()
+    n = 64 if curve == "mnt4_753" else 1024
+    pts, _ = oracle_points(curve, n if curve != "mnt4_753" else 64)
+    pts = pts.copy()
+    pts[5] = 0                                    # identity input
+    for dist in ("uniform", "zcash_like") if curve != "mnt4_753" else ("uniform",):
+        k = synth.scalars(curve, n, 41, dist)
+        want = oracle_msm_cached(curve, pts, k)
+        want_prefix = oracle_msm_cached(curve, pts[:n // 3], k[:n // 3])
+        for c in cs:
+            h = gz.PreparedPoints(curve, dev(pts), weighted=True, window_bits=c)
+            info = h.info()
+            assert info["weighted"] and info["window_bits"] == c
+            assert np.array_equal(host(h.msm(dev(k))), want), (dist, c)
+            assert np.array_equal(host(h.msm(dev(k[:n // 3]))), want_prefix), (dist, c)
+            h.release()
+
+
+def test_weighted_default_and_unweighted_prepare():
+    gz = require_cuda()
+    curve = "bn254"
+    pts, _ = oracle_points(curve, 1024)
+    k = synth.scalars(curve, 1024, 42)
+    want = oracle_msm_cached(curve, pts, k)
+    h = gz.PreparedPoints(curve, dev(pts))
+    assert h.info()["weighted"]
+    assert np.array_equal(host(h.msm(dev(k))), want)
+    h2 = gz.PreparedPoints(curve, dev(pts), weighted=False)
+    assert not h2.info()["weighted"]
+    assert np.array_equal(host(h2.msm(dev(k))), want)
