@@ -203,6 +203,124 @@ struct EC {
   }
 };
 
+// ---- warp-cooperative group law for latency-bound serial chains ----------
+// The window combination is a chain of (W-1)c doublings on ONE point; one
+// thread runs it at the latency of 9 dependent products per doubling.  Here
+// every lane of a warp holds the same point and lane q = lane & 3 computes the
+// q-th independent product of each dependency level of the formula, then the
+// products are broadcast with shuffles (warp-uniform control flow, no
+// divergence).  Critical path: 3 products per dbl-2008-s-1, 4 per add-2008-s.
+// This is the paper's cooperative-group idea applied at
+// the formula level instead of the limb level.
+template <class C>
+struct CoopEC {
+  static constexpr int N = C::N;
+  using Fp = F<C>;
+  using E = EC<C>;
+  using Xyzz = typename E::Xyzz;
+
+  GZ_DEV static void bcast(uint32_t d[N], const uint32_t s[N], int src) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) d[i] = __shfl_sync(0xffffffffu, s[i], src);
+  }
+  GZ_DEV static void pick(uint32_t d[N], int q, const uint32_t* a0, const uint32_t* a1, const uint32_t* a2,
+                          const uint32_t* a3) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) d[i] = q == 0 ? a0[i] : q == 1 ? a1[i] : q == 2 ? a2[i] : a3[i];
+  }
+  // one level: lane q computes r = x_q * y_q; results of lanes 0..k-1 broadcast
+  GZ_DEV static void level(uint32_t r[N], const uint32_t* x0, const uint32_t* y0, const uint32_t* x1,
+                           const uint32_t* y1, const uint32_t* x2, const uint32_t* y2, const uint32_t* x3,
+                           const uint32_t* y3) {
+    const int q = threadIdx.x & 3;
+    uint32_t x[N], y[N];
+    pick(x, q, x0, x1, x2, x3);
+    pick(y, q, y0, y1, y2, y3);
+    Fp::mul(r, x, y);
+  }
+
+  // P = 2P (all lanes hold P; identical result on every lane)
+  GZ_DEV static void dbl(Xyzz& P) {
+    uint32_t U[N], V[N], XX[N], W[N], S[N], MM[N], M[N], t[N], r[N];
+    Fp::dbl(U, P.Y);
+    // level 1: V = U^2, XX = X^2, (lane 2: ZZ^2 for a != 0)
+    level(r, U, U, P.X, P.X, P.ZZ, P.ZZ, U, U);
+    bcast(V, r, 0);
+    bcast(XX, r, 1);
+    Fp::add(M, XX, XX);
+    Fp::add(M, M, XX);
+    if constexpr (!C::A_ZERO) {
+      uint32_t z2[N];
+      bcast(z2, r, 2);
+      if constexpr (C::A_SMALL == 2) {
+        Fp::dbl(t, z2);
+      } else {
+        uint32_t a[N];
+#pragma unroll
+        for (int i = 0; i < N; ++i) a[i] = C::A_MONT(i);
+        Fp::mul(t, z2, a);
+      }
+      Fp::add(M, M, t);
+    }
+    // level 2: W = U V, S = X V, MM = M^2, ZZ3 = V ZZ
+    level(r, U, V, P.X, V, M, M, V, P.ZZ);
+    bcast(W, r, 0);
+    bcast(S, r, 1);
+    bcast(MM, r, 2);
+    bcast(P.ZZ, r, 3);
+    Fp::sub(t, MM, S);
+    Fp::sub(P.X, t, S);                 // X3 = M^2 - 2S
+    Fp::sub(t, S, P.X);
+    // level 3: M (S - X3), W Y, ZZZ3 = W ZZZ
+    level(r, M, t, W, P.Y, W, P.ZZZ, M, t);
+    bcast(t, r, 0);
+    bcast(U, r, 1);
+    bcast(P.ZZZ, r, 2);
+    Fp::sub(P.Y, t, U);                 // Y3 = M(S - X3) - W Y
+  }
+
+  // A += B, all cases (warp-uniform branches: every lane holds the same values)
+  GZ_DEV static void add(Xyzz& A, const Xyzz& B) {
+    if (E::is_inf(B)) return;
+    if (E::is_inf(A)) { A = B; return; }
+    uint32_t U1[N], S1[N], P[N], R[N], PP[N], RR[N], T1[N], T2[N], PPP[N], Q[N], t[N], r[N];
+    // level 1: U1 = X1 ZZ2, U2 = X2 ZZ1, S1 = Y1 ZZZ2, S2 = Y2 ZZZ1
+    level(r, A.X, B.ZZ, B.X, A.ZZ, A.Y, B.ZZZ, B.Y, A.ZZZ);
+    bcast(U1, r, 0);
+    bcast(P, r, 1);
+    bcast(S1, r, 2);
+    bcast(R, r, 3);
+    Fp::sub(P, P, U1);
+    Fp::sub(R, R, S1);
+    if (Fp::is_zero(P)) {
+      if (Fp::is_zero(R)) dbl(A);
+      else E::set_inf(A);
+      return;
+    }
+    // level 2: PP = P^2, RR = R^2, T1 = ZZ1 ZZ2, T2 = ZZZ1 ZZZ2
+    level(r, P, P, R, R, A.ZZ, B.ZZ, A.ZZZ, B.ZZZ);
+    bcast(PP, r, 0);
+    bcast(RR, r, 1);
+    bcast(T1, r, 2);
+    bcast(T2, r, 3);
+    // level 3: PPP = P PP, Q = U1 PP, ZZ3 = T1 PP
+    level(r, P, PP, U1, PP, T1, PP, P, PP);
+    bcast(PPP, r, 0);
+    bcast(Q, r, 1);
+    bcast(A.ZZ, r, 2);
+    Fp::sub(t, RR, PPP);
+    Fp::sub(t, t, Q);
+    Fp::sub(A.X, t, Q);                 // X3 = R^2 - PPP - 2Q
+    Fp::sub(t, Q, A.X);
+    // level 4: ZZZ3 = T2 PPP, S1 PPP, R (Q - X3)
+    level(r, T2, PPP, S1, PPP, R, t, T2, PPP);
+    bcast(A.ZZZ, r, 0);
+    bcast(S1, r, 1);
+    bcast(t, r, 2);
+    Fp::sub(A.Y, t, S1);                // Y3 = R(Q - X3) - S1 PPP
+  }
+};
+
 // ---- out-of-line versions for the cold kernels (merge, reduction, tail,
 // generators, diagnostics): one copy of each group-law body per TU keeps the
 // compile time and the instruction footprint bounded; only the bucket hot loop

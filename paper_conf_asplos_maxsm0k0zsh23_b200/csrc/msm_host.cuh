@@ -268,7 +268,7 @@ struct Impl {
     }
     profile_mark(prof, 4, s);
     // a7 + a8
-    k_tail<C><<<1, 1, 0, s>>>(U(p.o_win), p.Wb, p.c, (uint32_t*)call.out_partial, (uint32_t*)call.out_affine);
+    k_tail<C><<<1, 32, 0, s>>>(U(p.o_win), p.Wb, p.c, (uint32_t*)call.out_partial, (uint32_t*)call.out_affine);
     GZ_CHECK(cudaGetLastError());
     ++launches;
     profile_end(prof, U(p.o_offsets) + p.M, launches, p.c, s);

@@ -259,8 +259,16 @@ GZ_DEV uint32_t find_bucket(const uint32_t* __restrict__ off, uint32_t M, uint32
   return lo;
 }
 
+// CTAs per SM the hot loop is compiled for (registers: 128 / 168 / 255 per
+// thread).  BN254 fits 3 CTAs in 168 registers; for BLS12-381 forcing 3 CTAs
+// (166 regs) measured slower than the unconstrained 2 CTAs (85.6 % IMAD pipe).
 template <class C>
-__global__ void __launch_bounds__(128) k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off,
+struct AccumCfg {
+  static constexpr int MIN_CTAS = C::N <= 8 ? 3 : 1;
+};
+
+template <class C>
+__global__ void __launch_bounds__(128, AccumCfg<C>::MIN_CTAS) k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off,
                                                uint32_t M, const uint32_t* __restrict__ pts, int S,
                                                uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay) {
   using Fp = F<C>;
@@ -476,22 +484,25 @@ __global__ void __launch_bounds__(128) k_reduce_win(const uint32_t* __restrict__
 }
 
 // ----------------------------------------- a7 window combination + a8 output
-// Q = sum_t 2^(ct) W_t by Horner from the top window.  out_partial (XYZZ) and/or
-// out_affine (canonical) may be null.
+// Q = sum_t 2^(ct) W_t by Horner from the top window, on ONE warp with the
+// cooperative formulas (CoopEC).  Launch <<<1, 32>>>.  out_partial (XYZZ)
+// and/or out_affine (canonical) may be null.
 template <class C>
-__global__ void k_tail(const uint32_t* __restrict__ win_out, int W, int c, uint32_t* __restrict__ out_partial,
-                       uint32_t* __restrict__ out_affine) {
+__global__ void __launch_bounds__(32) k_tail(const uint32_t* __restrict__ win_out, int W, int c,
+                                             uint32_t* __restrict__ out_partial, uint32_t* __restrict__ out_affine) {
   using EC_ = EC<C>;
+  using CO = CoopEC<C>;
   constexpr int N = C::N;
-  if (threadIdx.x || blockIdx.x) return;
+  if (blockIdx.x) return;
   typename EC_::Xyzz Q;
   EC_::load(Q, win_out + (size_t)(W - 1) * 4 * N);
   for (int t = W - 2; t >= 0; --t) {
-    for (int k = 0; k < c; ++k) ec_dbl<C>(Q);
+    for (int k = 0; k < c; ++k) CO::dbl(Q);
     typename EC_::Xyzz X;
     EC_::load(X, win_out + (size_t)t * 4 * N);
-    ec_add<C>(Q, X);
+    CO::add(Q, X);
   }
+  if (threadIdx.x) return;
   if (EC_::is_inf(Q)) EC_::set_inf(Q);
   if (out_partial) EC_::store(out_partial, Q);
   if (out_affine) {
