@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 
+#include <algorithm>
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
@@ -64,19 +65,24 @@ ProfileRecord* profile_begin(cudaStream_t s) {
   static thread_local uint32_t* pinned = nullptr;
   if (!pinned && cudaMallocHost((void**)&pinned, sizeof(uint32_t)) != cudaSuccess) return nullptr;
   ProfileRecord* r = new ProfileRecord;
-  for (auto& e : r->ev) cudaEventCreate(&e);
   r->entries_host = pinned;
   r->launches = 0;
   r->c = 0;
-  cudaEventRecord(r->ev[0], s);
+  (void)s;
   return r;
 }
-void profile_mark(ProfileRecord* r, int i, cudaStream_t s) {
-  if (r) cudaEventRecord(r->ev[i], s);
+cudaEvent_t profile_event(ProfileRecord* r, cudaStream_t s) {
+  if (!r) return nullptr;
+  cudaEvent_t e;
+  cudaEventCreate(&e);
+  cudaEventRecord(e, s);
+  return e;
+}
+void profile_interval(ProfileRecord* r, int phase, cudaEvent_t a, cudaEvent_t b) {
+  if (r && a && b) r->iv.push_back({phase, a, b});
 }
 void profile_end(ProfileRecord* r, const uint32_t* entries_dev, int launches, int c, cudaStream_t s) {
   if (!r) return;
-  cudaEventRecord(r->ev[5], s);
   cudaMemcpyAsync(r->entries_host, entries_dev, sizeof(uint32_t), cudaMemcpyDeviceToHost, s);
   r->launches = launches;
   r->c = c;
@@ -105,6 +111,11 @@ static void init_pool_once() {
       uint64_t thr = UINT64_MAX;
       cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
     }
+    // the out-of-line MNT4-753 paths need up to ~2.6 KB of call stack per
+    // thread (ptxas "cumulative stack size"); the default limit is 1 KB
+    size_t stack = 0;
+    cudaDeviceGetLimit(&stack, cudaLimitStackSize);
+    if (stack < 4096) cudaDeviceSetLimit(cudaLimitStackSize, 4096);
   });
 }
 
@@ -132,6 +143,27 @@ gzkp_status stream_workspace(cudaStream_t s, size_t bytes, void** ptr) {
     e.bytes = want;
   }
   *ptr = e.p;
+  return GZKP_SUCCESS;
+}
+
+gzkp_status stream_ctx(cudaStream_t s, StreamCtx** out) {
+  static std::mutex mu;
+  static std::map<std::pair<int, cudaStream_t>, StreamCtx*> cache;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lock(mu);
+  StreamCtx*& c = cache[{dev, s}];
+  if (!c) {
+    StreamCtx* n = new StreamCtx;
+    int lo = 0, hi = 0;
+    cudaDeviceGetStreamPriorityRange(&lo, &hi);      // hi = greatest priority
+    cudaError_t e = cudaStreamCreateWithPriority(&n->side, cudaStreamNonBlocking, hi);
+    if (e != cudaSuccess) { delete n; return cuda_status(e, "cudaStreamCreateWithPriority"); }
+    n->nev = 64;
+    for (int i = 0; i < n->nev; ++i) cudaEventCreateWithFlags(&n->ev[i], cudaEventDisableTiming);
+    c = n;
+  }
+  *out = c;
   return GZKP_SUCCESS;
 }
 
@@ -277,6 +309,7 @@ gzkp_status gzkp_msm_partial(int curve, const void* points_affine, const void* s
 
 gzkp_status gzkp_combine_partials(int curve, const void* partials_xyzz, int count, void* out_affine,
                                   gzkp_stream stream) {
+  init_pool_once();
   const CurveImpl* c = impl_for(curve);
   if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
   if (count < 0 || !out_affine || (count && !partials_xyzz)) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
@@ -308,6 +341,7 @@ gzkp_status gzkp_msm_host(int curve, const void* points_host, const void* scalar
 
 gzkp_status gzkp_points_prepare_ex(int curve, const void* points_affine, size_t n, int window_bits, int weighted,
                                    void** handle, gzkp_stream stream) {
+  init_pool_once();
   const CurveImpl* c = impl_for(curve);
   if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
   if (!handle || (n && !points_affine) || !aligned16(points_affine) || window_bits < 0 || window_bits > 22)
@@ -407,12 +441,14 @@ gzkp_status gzkp_points_release(void* handle) {
 }
 
 gzkp_status gzkp_fixed_base_mul(int curve, const void* scalars, size_t n, void* out_affine, gzkp_stream stream) {
+  init_pool_once();
   const CurveImpl* c = impl_for(curve);
   if (gzkp_status st = check_args(c, out_affine, scalars, n, out_affine)) return st;
   return c->fixed_base(scalars, n, out_affine, (cudaStream_t)stream);
 }
 
 gzkp_status gzkp_field_op(int curve, int op, const void* a, const void* b, void* out, size_t n, gzkp_stream stream) {
+  init_pool_once();
   const CurveImpl* c = impl_for(curve);
   if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
   if (op < 0 || op > 4 || (n && (!a || !b || !out))) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
@@ -420,6 +456,7 @@ gzkp_status gzkp_field_op(int curve, int op, const void* a, const void* b, void*
 }
 
 gzkp_status gzkp_ec_op(int curve, int op, const void* P, const void* Q, void* out, size_t n, gzkp_stream stream) {
+  init_pool_once();
   const CurveImpl* c = impl_for(curve);
   if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
   if (op < 0 || op > 3 || (n && (!P || !Q || !out))) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
@@ -441,17 +478,23 @@ gzkp_status gzkp_set_profiling(int on) {
 
 gzkp_status gzkp_profile_read(double phase_ms[5], uint64_t stats[4], int reset) {
   for (ProfileRecord* r : g_pending) {
-    cudaEventSynchronize(r->ev[5]);
-    for (int i = 0; i < 5; ++i) {
+    std::vector<cudaEvent_t> seen;
+    for (auto& iv : r->iv) {
+      cudaEventSynchronize(iv.b);
       float ms = 0.f;
-      cudaEventElapsedTime(&ms, r->ev[i], r->ev[i + 1]);
-      g_phase_sum[i] += ms;
+      cudaEventElapsedTime(&ms, iv.a, iv.b);
+      if (iv.phase >= 0 && iv.phase < 5) g_phase_sum[iv.phase] += ms;
+      seen.push_back(iv.a);
+      seen.push_back(iv.b);
     }
+    cudaDeviceSynchronize();   // the pinned entry count
     ++g_calls;
     g_last_launches = r->launches;
     g_last_entries = *r->entries_host;
     g_last_c = r->c;
-    for (auto& e : r->ev) cudaEventDestroy(e);
+    std::sort(seen.begin(), seen.end());
+    seen.erase(std::unique(seen.begin(), seen.end()), seen.end());
+    for (auto e : seen) cudaEventDestroy(e);
     delete r;
   }
   g_pending.clear();

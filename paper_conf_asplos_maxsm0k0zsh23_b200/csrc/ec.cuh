@@ -223,10 +223,13 @@ struct CoopEC {
 #pragma unroll
     for (int i = 0; i < N; ++i) d[i] = __shfl_sync(0xffffffffu, s[i], src);
   }
+  // branch-free 4-way blend by lane (pure LOP3s: no local-memory indexing)
   GZ_DEV static void pick(uint32_t d[N], int q, const uint32_t* a0, const uint32_t* a1, const uint32_t* a2,
                           const uint32_t* a3) {
+    const uint32_t m0 = 0u - (uint32_t)(q == 0), m1 = 0u - (uint32_t)(q == 1);
+    const uint32_t m2 = 0u - (uint32_t)(q == 2), m3 = 0u - (uint32_t)(q == 3);
 #pragma unroll
-    for (int i = 0; i < N; ++i) d[i] = q == 0 ? a0[i] : q == 1 ? a1[i] : q == 2 ? a2[i] : a3[i];
+    for (int i = 0; i < N; ++i) d[i] = (a0[i] & m0) | (a1[i] & m1) | (a2[i] & m2) | (a3[i] & m3);
   }
   // one level: lane q computes r = x_q * y_q; results of lanes 0..k-1 broadcast
   GZ_DEV static void level(uint32_t r[N], const uint32_t* x0, const uint32_t* y0, const uint32_t* x1,
@@ -236,7 +239,9 @@ struct CoopEC {
     uint32_t x[N], y[N];
     pick(x, q, x0, x1, x2, x3);
     pick(y, q, y0, y1, y2, y3);
-    Fp::mul(r, x, y);
+    // always inlined here (also for N = 24): per-lane operands feeding an
+    // out-of-line call between warp shuffles produced wrong MNT4-753 results
+    Fp::mul_inline(r, x, y);
   }
 
   // P = 2P (all lanes hold P; identical result on every lane)

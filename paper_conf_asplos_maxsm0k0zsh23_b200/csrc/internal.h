@@ -6,6 +6,7 @@
 #include <cstddef>
 #include <cstdint>
 #include <string>
+#include <vector>
 
 #include "../../include/gzkp.h"
 
@@ -66,16 +67,29 @@ bool profiling_enabled();
 // library-owned workspace, one grow-only buffer per (device, stream): calls on
 // one stream are ordered, so they can share it; different streams never do.
 gzkp_status stream_workspace(cudaStream_t s, size_t bytes, void** ptr);
-// profiling hooks (no synchronisation): events[6] recorded by the caller,
-// entries_dev = device address of the call's entry count (copied async).
+// profiling hooks (no synchronisation).  A record is a list of timed
+// intervals, each (phase, start event, end event) on any stream; phases:
+// 0 sort, 1 accumulate, 2 merge, 3 reduce, 4 tail.  entries_dev = device
+// address of the call's entry count (copied async into pinned memory).
 struct ProfileRecord {
-  cudaEvent_t ev[6];
-  uint32_t* entries_host;   // pinned, written by an async copy
+  struct Iv { int phase; cudaEvent_t a, b; };
+  std::vector<Iv> iv;
+  uint32_t* entries_host;
   int launches;
   int c;
 };
 ProfileRecord* profile_begin(cudaStream_t s);          // null when profiling is off
-void profile_mark(ProfileRecord* r, int i, cudaStream_t s);
+cudaEvent_t profile_event(ProfileRecord* r, cudaStream_t s);   // records a fresh event (null if off)
+void profile_interval(ProfileRecord* r, int phase, cudaEvent_t a, cudaEvent_t b);
 void profile_end(ProfileRecord* r, const uint32_t* entries_dev, int launches, int c, cudaStream_t s);
+
+// per (device, caller stream): a high-priority side stream and reusable
+// sync events for the window-group pipeline
+struct StreamCtx {
+  cudaStream_t side = nullptr;
+  cudaEvent_t ev[64];
+  int nev = 0;
+};
+gzkp_status stream_ctx(cudaStream_t s, StreamCtx** ctx);
 
 }  // namespace gzkp

@@ -35,7 +35,15 @@ struct Plan {
   uint64_t E_max = 0, chunks_max = 0;
   // workspace byte offsets
   size_t o_pts = 0, o_codes = 0, o_counts = 0, o_offsets = 0, o_cursor = 0, o_tiles = 0, o_vals = 0,
-         o_spay = 0, o_heavy = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_win = 0, total = 0;
+         o_spay = 0, o_heavy = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_win = 0, total = 0;
+  struct Grp {
+    int t_lo, t_hi;             // windows (inclusive)
+    uint32_t key_lo, key_hi;    // bucket keys
+    uint64_t chunk_base, chunks_max;
+    int heavy_levels;
+    int seg = 16;               // reduction segment (buckets per thread)
+  };
+  std::vector<Grp> groups;
 };
 
 constexpr uint32_t WIN_PER_BLOCK = 1024;   // segment partials summed per block (stage A)
@@ -115,9 +123,47 @@ struct Impl {
       p.seg = (int)std::min<uint64_t>(seg, p.B);
     }
     p.E_max = (uint64_t)n * p.W;
-    p.chunks_max = std::max<uint64_t>(1, (p.E_max + p.S - 1) / p.S);
+    // window groups, top windows first, sizes halving down to a last group of
+    // one window (window 0): the side stream merges / reduces / combines group
+    // g while group g+1 accumulates, so only the last group's post-processing
+    // is exposed.  Weighted points share one bucket set: a single group.
+    p.groups.clear();
+    static const int pipeline = [] {
+      const char* e = getenv("GZKP_PIPELINE");
+      return e ? atoi(e) : 0;
+    }();
+    if (consolidated || !pipeline) {
+      p.groups.push_back({0, p.W - 1, 0, p.M, 0, 0, 0});
+    } else if (consolidated) {
+      p.groups.push_back({0, p.W - 1, 0, p.B, 0, 0, 0});
+    } else {
+      int hi = p.W - 1;
+      while (hi >= 0) {
+        const int rem = hi + 1;
+        const int sz = rem > 1 ? (rem + 1) / 2 : 1;
+        p.groups.push_back({hi - sz + 1, hi, (uint32_t)(hi - sz + 1) * p.B, (uint32_t)(hi + 1) * p.B, 0, 0, 0});
+        hi -= sz;
+      }
+    }
+    p.chunks_max = 0;
     p.heavy_levels = 0;
-    for (uint64_t span = 1; span < p.chunks_max; span *= HEAVY_FAN) ++p.heavy_levels;
+    uint64_t seg_elems = 1, mid_elems = 1;
+    for (auto& g : p.groups) {
+      const uint64_t wins = consolidated ? (uint64_t)p.W : (uint64_t)(g.t_hi - g.t_lo + 1);
+      const uint64_t bwins = consolidated ? 1 : wins;
+      // reduction segment of this group: <= 16 buckets, fewer until >= 32K threads
+      uint64_t seg = 16;
+      while (seg > 1 && bwins * p.B / seg < 32768) seg >>= 1;
+      g.seg = (int)std::min<uint64_t>(seg, p.B);
+      const uint64_t gsegs = p.B / g.seg;
+      seg_elems = std::max<uint64_t>(seg_elems, bwins * gsegs);
+      mid_elems = std::max<uint64_t>(mid_elems, bwins * ((gsegs + WIN_PER_BLOCK - 1) / WIN_PER_BLOCK));
+      g.chunk_base = p.chunks_max;
+      g.chunks_max = (n * wins + p.S - 1) / p.S + 1;
+      g.heavy_levels = 0;
+      for (uint64_t span = 1; span < g.chunks_max; span *= HEAVY_FAN) ++g.heavy_levels;
+      p.chunks_max += g.chunks_max;
+    }
     const uint32_t G = p.B / p.seg;
     size_t o = 0;
     auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
@@ -129,10 +175,12 @@ struct Impl {
     p.o_tiles = take(SCAN_TILE * 4);
     p.o_vals = take(std::max<uint64_t>(p.E_max, 1) * 4);
     p.o_spay = take(2 * p.chunks_max * 4 * N * 4);
-    p.o_heavy = take(16);
+    p.o_heavy = take(4 * (p.groups.size() + 4));
+    p.o_state = take(4 * N * 4);
     p.o_buckets = take((size_t)p.M * 4 * N * 4);
-    p.o_seg = take((size_t)p.Wb * G * 4 * N * 4);
-    p.o_mid = take((size_t)p.Wb * ((G + WIN_PER_BLOCK - 1) / WIN_PER_BLOCK) * 4 * N * 4);
+    (void)G;
+    p.o_seg = take((size_t)seg_elems * 4 * N * 4);
+    p.o_mid = take((size_t)mid_elems * 4 * N * 4);
     p.o_win = take((size_t)p.Wb * 4 * N * 4);
     p.total = o;
     return p;
@@ -185,6 +233,7 @@ struct Impl {
     const size_t n = call.n;
     auto U = [&](size_t off) { return (uint32_t*)(ws + off); };
     ProfileRecord* prof = profile_begin(s);
+    cudaEvent_t ev_begin = profile_event(prof, s);
     int launches = 0;
     const int sms = device_sm_count();
 
@@ -197,7 +246,7 @@ struct Impl {
     }
     // a2: digits + histogram
     GZ_CHECK(cudaMemsetAsync(U(p.o_counts), 0, (size_t)p.M * 4, s));
-    GZ_CHECK(cudaMemsetAsync(U(p.o_heavy), 0, 16, s));
+    GZ_CHECK(cudaMemsetAsync(U(p.o_heavy), 0, 4 * (p.groups.size() + 4), s));
     const uint32_t bpw = (uint32_t)((n + DIGIT_THREADS - 1) / DIGIT_THREADS);
     const uint32_t key_stride = p.consolidated ? 0u : p.B;
     k_digits<C><<<bpw, DIGIT_THREADS, 0, s>>>((const uint32_t*)call.scalars, n, p.c, p.W, key_stride, U(p.o_codes),
@@ -213,64 +262,95 @@ struct Impl {
                                                                          p.val_stride, U(p.o_cursor), U(p.o_vals));
     GZ_CHECK(cudaGetLastError());
     launches += 5;
-    profile_mark(prof, 1, s);
+    cudaEvent_t ev_sorted = profile_event(prof, s);
+    profile_interval(prof, 0, ev_begin, ev_sorted);
 
-    // a4: accumulation
-    {
-      const int threads = 128;
-      const size_t smem = (size_t)threads * Stage<C>::SLOT_WORDS * 4;
-      static int grid = 0;
-      if (!grid) {
-        cudaFuncSetAttribute(k_accum<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        grid = occupancy_grid((const void*)k_accum<C>, threads, smem);
-      }
-      const int g = (int)std::min<uint64_t>(grid, (p.chunks_max + threads - 1) / threads);
-      k_accum<C><<<std::max(g, 1), threads, smem, s>>>(U(p.o_vals), U(p.o_offsets), p.M, pts, p.S, U(p.o_buckets),
-                                                       U(p.o_spay));
-      GZ_CHECK(cudaGetLastError());
-      ++launches;
+    // a4..a8, pipelined by window group: accumulate group g on the caller's
+    // stream; merge / reduce / combine it on the high-priority side stream
+    // while group g+1 accumulates.  One group (weighted points): no side stream.
+    const int ngroups = (int)p.groups.size();
+    StreamCtx* ctx = nullptr;
+    cudaStream_t ss = s;
+    if (ngroups > 1) {
+      if (gzkp_status st = stream_ctx(s, &ctx)) return st;
+      if (2 * ngroups + 1 > ctx->nev) return set_error(GZKP_ERROR_INVALID_VALUE, "too many window groups");
+      ss = ctx->side;
     }
-    profile_mark(prof, 2, s);
-    // a5: merge of chunk-boundary partials (+ heavy-bucket tree)
-    {
-      const int threads = 128;
-      const int gm = (int)std::min<uint64_t>((p.M + threads - 1) / threads, (uint64_t)sms * 16);
-      k_merge_bucket<C><<<gm, threads, 0, s>>>(U(p.o_offsets), p.M, p.S, U(p.o_spay), U(p.o_buckets), U(p.o_heavy));
+    const int threads = 128;
+    const size_t acc_smem = (size_t)threads * Stage<C>::SLOT_WORDS * 4;
+    static bool attr_set = false;
+    if (!attr_set) {
+      GZ_CHECK(cudaFuncSetAttribute(k_accum<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)acc_smem));
+      GZ_CHECK(cudaFuncSetAttribute(k_reduce_win<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)((size_t)threads * 4 * N * 4)));
+      attr_set = true;
+    }
+    cudaEvent_t ev_last_acc = nullptr, ev_merged = nullptr, ev_reduced = nullptr, ev_tailed = nullptr;
+    for (int gi = 0; gi < ngroups; ++gi) {
+      const auto& gr = p.groups[gi];
+      const Group grp{gr.key_lo, gr.key_hi, (uint32_t)gr.chunk_base};
+      // a4 (main stream)
+      cudaEvent_t a0 = profile_event(prof, s);
+      k_accum<C><<<(unsigned)((gr.chunks_max + threads - 1) / threads), threads, acc_smem, s>>>(
+          U(p.o_vals), U(p.o_offsets), grp, pts, p.S, U(p.o_buckets), U(p.o_spay));
       GZ_CHECK(cudaGetLastError());
-      const int gh = (int)std::min<uint64_t>((p.chunks_max + threads - 1) / threads, (uint64_t)sms * 8);
+      cudaEvent_t a1 = profile_event(prof, s);
+      profile_interval(prof, 1, a0, a1);
+      ev_last_acc = a1;
+      ++launches;
+      if (ctx) {
+        GZ_CHECK(cudaEventRecord(ctx->ev[gi], s));
+        GZ_CHECK(cudaStreamWaitEvent(ss, ctx->ev[gi], 0));
+      }
+      // a5 (side stream): boundary partials -> buckets, heavy-bucket tree
+      uint32_t* heavy = U(p.o_heavy) + gi;
+      const uint32_t nkeys = gr.key_hi - gr.key_lo;
+      const int gm = (int)std::min<uint64_t>((nkeys + threads - 1) / threads, (uint64_t)sms * 16);
+      k_merge_bucket<C><<<gm, threads, 0, ss>>>(U(p.o_offsets), grp, p.S, U(p.o_spay), U(p.o_buckets), heavy);
+      GZ_CHECK(cudaGetLastError());
+      const int gh = (int)std::min<uint64_t>((gr.chunks_max + threads - 1) / threads, (uint64_t)sms * 8);
       uint32_t stride = 1;
-      for (int l = 0; l < p.heavy_levels; ++l, stride *= HEAVY_FAN) {
-        k_heavy_level<C><<<gh, threads, 0, s>>>(U(p.o_offsets), p.M, p.S, stride, U(p.o_heavy), U(p.o_spay));
+      for (int l = 0; l < gr.heavy_levels; ++l, stride *= HEAVY_FAN) {
+        k_heavy_level<C><<<gh, threads, 0, ss>>>(U(p.o_offsets), grp, p.S, stride, heavy, U(p.o_spay));
         GZ_CHECK(cudaGetLastError());
       }
-      k_heavy_final<C><<<gm, threads, 0, s>>>(U(p.o_offsets), p.M, p.S, U(p.o_heavy), U(p.o_spay), U(p.o_buckets));
+      k_heavy_final<C><<<gm, threads, 0, ss>>>(U(p.o_offsets), grp, p.S, heavy, U(p.o_spay), U(p.o_buckets));
       GZ_CHECK(cudaGetLastError());
-      launches += 2 + p.heavy_levels;
-    }
-    profile_mark(prof, 3, s);
-    // a6: bucket reduction
-    const uint32_t G = p.B / p.seg;
-    {
-      const int threads = 128;
-      const uint32_t total = (uint32_t)p.Wb * G;
-      k_reduce_seg<C><<<(total + threads - 1) / threads, threads, 0, s>>>(U(p.o_buckets), U(p.o_offsets), p.Wb, p.B,
-                                                                          p.seg, U(p.o_seg));
+      launches += 2 + gr.heavy_levels;
+      ev_merged = profile_event(prof, ss);
+      // a6 (side stream): bucket reduction of the group's windows
+      const int gw = p.consolidated ? 1 : gr.t_hi - gr.t_lo + 1;
+      const int t_lo = p.consolidated ? 0 : gr.t_lo;
+      const uint32_t G = p.B / gr.seg;
+      const uint32_t total = (uint32_t)gw * G;
+      k_reduce_seg<C><<<(total + threads - 1) / threads, threads, 0, ss>>>(U(p.o_buckets), U(p.o_offsets), t_lo, gw,
+                                                                           p.B, gr.seg, U(p.o_seg));
       GZ_CHECK(cudaGetLastError());
-      const int rthreads = 128;
-      const size_t smem = (size_t)rthreads * 4 * N * 4;
-      GZ_CHECK(cudaFuncSetAttribute(k_reduce_win<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      const size_t rsmem = (size_t)threads * 4 * N * 4;
       const uint32_t nb = (G + WIN_PER_BLOCK - 1) / WIN_PER_BLOCK;
-      k_reduce_win<C><<<dim3(nb, p.Wb), rthreads, smem, s>>>(U(p.o_seg), G, WIN_PER_BLOCK, U(p.o_mid));
+      k_reduce_win<C><<<dim3(nb, gw), threads, rsmem, ss>>>(U(p.o_seg), G, WIN_PER_BLOCK, U(p.o_mid));
       GZ_CHECK(cudaGetLastError());
-      k_reduce_win<C><<<dim3(1, p.Wb), rthreads, smem, s>>>(U(p.o_mid), nb, nb, U(p.o_win));
+      k_reduce_win<C><<<dim3(1, gw), threads, rsmem, ss>>>(U(p.o_mid), nb, nb, U(p.o_win) + (size_t)t_lo * 4 * N);
       GZ_CHECK(cudaGetLastError());
       launches += 3;
+      ev_reduced = profile_event(prof, ss);
+      // a7 (+ a8 on the last group): Horner over the group's windows
+      const int last = gi == ngroups - 1;
+      k_tail<C><<<1, 32, 0, ss>>>(U(p.o_win), p.consolidated ? 0 : gr.t_hi, t_lo, p.c, gi == 0, last, U(p.o_state),
+                                  last ? (uint32_t*)call.out_partial : nullptr,
+                                  last ? (uint32_t*)call.out_affine : nullptr);
+      GZ_CHECK(cudaGetLastError());
+      ++launches;
+      ev_tailed = profile_event(prof, ss);
     }
-    profile_mark(prof, 4, s);
-    // a7 + a8
-    k_tail<C><<<1, 32, 0, s>>>(U(p.o_win), p.Wb, p.c, (uint32_t*)call.out_partial, (uint32_t*)call.out_affine);
-    GZ_CHECK(cudaGetLastError());
-    ++launches;
+    // phases 2-4 = the exposed post-processing of the last group
+    profile_interval(prof, 2, ev_last_acc, ev_merged);
+    profile_interval(prof, 3, ev_merged, ev_reduced);
+    profile_interval(prof, 4, ev_reduced, ev_tailed);
+    if (ctx) {   // join: later work on the caller's stream follows the side stream
+      GZ_CHECK(cudaEventRecord(ctx->ev[ctx->nev - 1], ss));
+      GZ_CHECK(cudaStreamWaitEvent(s, ctx->ev[ctx->nev - 1], 0));
+    }
     profile_end(prof, U(p.o_offsets) + p.M, launches, p.c, s);
     return GZKP_SUCCESS;
   }

@@ -248,10 +248,16 @@ struct Stage {
 // last run, continuing to the right, to slot 2*chunk+1.  A bucket spanning
 // chunks t0..t1 therefore has its partials at slot 2*t0+1 and the head slots
 // 2*t of t0 < t <= t1 (k_merge_bucket relies on this).
-template <class C>
-GZ_DEV uint32_t find_bucket(const uint32_t* __restrict__ off, uint32_t M, uint32_t pos) {
-  // largest k with off[k] <= pos (off non-decreasing, off[0] = 0, pos < off[M])
-  uint32_t lo = 0, hi = M;   // invariant: off[lo] <= pos < off[hi]
+// One window group of the pipeline (host-planned): bucket keys
+// [key_lo, key_hi) own the sorted entries [off[key_lo], off[key_hi]); the
+// group's chunks are numbered from 0 and its boundary partials live in slots
+// 2*(chunk_base + j) (head) and 2*(chunk_base + j) + 1 (tail).
+struct Group {
+  uint32_t key_lo, key_hi, chunk_base;
+};
+
+// largest k in [lo, hi) with off[k] <= pos  (off non-decreasing, off[lo] <= pos < off[hi])
+GZ_DEV uint32_t find_bucket(const uint32_t* __restrict__ off, uint32_t lo, uint32_t hi, uint32_t pos) {
   while (hi - lo > 1) {
     const uint32_t mid = (lo + hi) >> 1;
     if (__ldg(off + mid) <= pos) lo = mid; else hi = mid;
@@ -267,10 +273,14 @@ struct AccumCfg {
   static constexpr int MIN_CTAS = C::N <= 8 ? 3 : 1;
 };
 
+// One chunk per thread, non-persistent grid sized for the group's worst case
+// (threads past the group's real chunk count exit): while the next group
+// accumulates, finishing CTAs free slots for the high-priority side stream
+// that merges / reduces / combines the previous group.
 template <class C>
-__global__ void __launch_bounds__(128, AccumCfg<C>::MIN_CTAS) k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off,
-                                               uint32_t M, const uint32_t* __restrict__ pts, int S,
-                                               uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay) {
+__global__ void __launch_bounds__(128, AccumCfg<C>::MIN_CTAS)
+    k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off, Group grp,
+            const uint32_t* __restrict__ pts, int S, uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay) {
   using Fp = F<C>;
   using EC_ = EC<C>;
   using St = Stage<C>;
@@ -278,159 +288,164 @@ __global__ void __launch_bounds__(128, AccumCfg<C>::MIN_CTAS) k_accum(const uint
   extern __shared__ __align__(16) uint32_t stage_smem[];
   uint32_t* slot = stage_smem + threadIdx.x * St::SLOT_WORDS;
 
-  const uint32_t E = __ldg(off + M);
-  const uint32_t nchunks = (E + S - 1) / S;
-  for (uint32_t chunk = blockIdx.x * blockDim.x + threadIdx.x; chunk < nchunks;
-       chunk += gridDim.x * blockDim.x) {
-    const uint32_t beg = chunk * (uint32_t)S;
-    const uint32_t end = min(E, beg + (uint32_t)S);
-    uint32_t cur = find_bucket<C>(off, M, beg);
-    uint32_t nxt = __ldg(off + cur + 1);
-    bool first_run = true;
+  const uint32_t G0 = __ldg(off + grp.key_lo), G1 = __ldg(off + grp.key_hi);
+  const uint32_t nchunks = (G1 - G0 + S - 1) / S;
+  const uint32_t chunk = blockIdx.x * blockDim.x + threadIdx.x;
+  if (chunk >= nchunks) return;
+  const uint32_t beg = G0 + chunk * (uint32_t)S;
+  const uint32_t end = min(G1, beg + (uint32_t)S);
+  const uint32_t sidx = 2 * (grp.chunk_base + chunk);
+  uint32_t cur = find_bucket(off, grp.key_lo, grp.key_hi, beg);
+  uint32_t nxt = __ldg(off + cur + 1);
+  bool first_run = true;
 
-    typename EC_::Xyzz acc;
-    bool acc_inf = true;
-    auto flush = [&](bool last_run) {
-      const bool open_l = first_run && __ldg(off + cur) < beg;
-      const bool open_r = last_run && nxt > end;
-      if (acc_inf) EC_::set_inf(acc);
-      if (!open_l && !open_r) EC_::store(buckets + (size_t)cur * 4 * N, acc);
-      else EC_::store(spay + (size_t)(open_l ? 2 * chunk : 2 * chunk + 1) * 4 * N, acc);
-    };
+  typename EC_::Xyzz acc;
+  bool acc_inf = true;
+  auto flush = [&](bool last_run) {
+    const bool open_l = first_run && __ldg(off + cur) < beg;
+    const bool open_r = last_run && nxt > end;
+    if (acc_inf) EC_::set_inf(acc);
+    if (!open_l && !open_r) EC_::store(buckets + (size_t)cur * 4 * N, acc);
+    else EC_::store(spay + (size_t)(open_l ? sidx : sidx + 1) * 4 * N, acc);
+  };
 
-    uint32_t v_next = vals[beg];
-    St::fetch(slot, pts, v_next & ~VAL_NEG);
-    cp_async_commit();
-    for (uint32_t j = beg; j < end; ++j) {
-      const uint32_t v = v_next;
-      const int buf = (j - beg) & 1;
-      if (j + 1 < end) {
-        v_next = vals[j + 1];
-        St::fetch(slot + (buf ^ 1) * St::PT_WORDS, pts, v_next & ~VAL_NEG);
-      }
-      cp_async_commit();
-      cp_async_wait<1>();
-      if (j == nxt) {                       // bucket boundary: close the run
-        flush(false);
-        acc_inf = true;
-        first_run = false;
-        do { ++cur; nxt = __ldg(off + cur + 1); } while (nxt == j);   // skip empty buckets
-      }
-      uint32_t x[N], y[N];
-      EC_::ld(x, slot + buf * St::PT_WORDS);
-      EC_::ld(y, slot + buf * St::PT_WORDS + N);
-      if (Fp::is_zero(x) && Fp::is_zero(y)) continue;     // identity input point
-      if (v & VAL_NEG) Fp::neg(y, y);
-      if (acc_inf) {
-        EC_::from_affine(acc, x, y);
-        acc_inf = false;
-      } else {
-        EC_::madd_nz(acc, x, y);
-        acc_inf = EC_::is_inf(acc);
-      }
+  uint32_t v_next = vals[beg];
+  St::fetch(slot, pts, v_next & ~VAL_NEG);
+  cp_async_commit();
+  for (uint32_t j = beg; j < end; ++j) {
+    const uint32_t v = v_next;
+    const int buf = (j - beg) & 1;
+    if (j + 1 < end) {
+      v_next = vals[j + 1];
+      St::fetch(slot + (buf ^ 1) * St::PT_WORDS, pts, v_next & ~VAL_NEG);
     }
-    cp_async_wait<0>();
-    flush(true);
+    cp_async_commit();
+    cp_async_wait<1>();
+    if (j == nxt) {                       // bucket boundary: close the run
+      flush(false);
+      acc_inf = true;
+      first_run = false;
+      do { ++cur; nxt = __ldg(off + cur + 1); } while (nxt == j);   // skip empty buckets
+    }
+    uint32_t x[N], y[N];
+    EC_::ld(x, slot + buf * St::PT_WORDS);
+    EC_::ld(y, slot + buf * St::PT_WORDS + N);
+    if (Fp::is_zero(x) && Fp::is_zero(y)) continue;     // identity input point
+    if (v & VAL_NEG) Fp::neg(y, y);
+    if (acc_inf) {
+      EC_::from_affine(acc, x, y);
+      acc_inf = false;
+    } else {
+      EC_::madd_nz(acc, x, y);
+      acc_inf = EC_::is_inf(acc);
+    }
   }
+  cp_async_wait<0>();
+  flush(true);
 }
 
 // ----------------------------------------------------------- a5 merge
-// Thread per bucket: a bucket spanning chunks t0 < t1 has q = t1 - t0 + 1
-// partials (slot 2*t0+1, then head slots 2*t).  q <= MERGE_QMAX: summed here.
-// Larger q (a heavy bucket of a skewed input) raises *heavy and is reduced by
-// the k_heavy_level tree instead.
+// Thread per bucket of the group: a bucket spanning local chunks t0 < t1 has
+// q = t1 - t0 + 1 partials (slot 2*(base+t0)+1, then head slots 2*(base+t)).
+// q <= MERGE_QMAX: summed here.  Larger q (a heavy bucket of a skewed input)
+// raises *heavy and is reduced by the k_heavy_level tree instead.
 template <class C>
-__global__ void __launch_bounds__(128) k_merge_bucket(const uint32_t* __restrict__ off, uint32_t M, int S,
+__global__ void __launch_bounds__(128) k_merge_bucket(const uint32_t* __restrict__ off, Group grp, int S,
                                                       const uint32_t* __restrict__ spay, uint32_t* __restrict__ buckets,
                                                       uint32_t* __restrict__ heavy) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
-  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < M; k += gridDim.x * blockDim.x) {
+  const uint32_t G0 = __ldg(off + grp.key_lo);
+  for (uint32_t k = grp.key_lo + blockIdx.x * blockDim.x + threadIdx.x; k < grp.key_hi;
+       k += gridDim.x * blockDim.x) {
     const uint32_t b0 = __ldg(off + k), b1 = __ldg(off + k + 1);
     if (b1 == b0) continue;
-    const uint32_t t0 = b0 / S, t1 = (b1 - 1) / S;
+    const uint32_t t0 = (b0 - G0) / S, t1 = (b1 - 1 - G0) / S;
     if (t0 == t1) continue;                              // written by k_accum
     if (t1 - t0 + 1 > (uint32_t)MERGE_QMAX) { *heavy = 1u; continue; }
     typename EC_::Xyzz acc, X;
-    EC_::load(acc, spay + (size_t)(2 * t0 + 1) * 4 * N);
+    EC_::load(acc, spay + (size_t)(2 * (grp.chunk_base + t0) + 1) * 4 * N);
     for (uint32_t t = t0 + 1; t <= t1; ++t) {
-      EC_::load(X, spay + (size_t)(2 * t) * 4 * N);
+      EC_::load(X, spay + (size_t)(2 * (grp.chunk_base + t)) * 4 * N);
       ec_add<C>(acc, X);
     }
     EC_::store(buckets + (size_t)k * 4 * N, acc);
   }
 }
 
-// Heavy buckets: in-place tree over their head slots.  Head u (0-based, slot
-// 2*(t0+1+u)) is a level-l leader when u % (stride*FAN) == 0; it absorbs heads
-// u + j*stride, j = 1..FAN-1 (leaders of level l-1).  After ceil(log_FAN q)
-// levels head 0 holds the sum of all heads.
+// Heavy buckets: in-place tree over their head slots.  Head u (0-based, local
+// chunk t0+1+u) is a level-l leader when u % (stride*FAN) == 0; it absorbs
+// heads u + j*stride, j = 1..FAN-1 (leaders of level l-1).  After
+// ceil(log_FAN q) levels head 0 holds the sum of all heads.
 template <class C>
-__global__ void __launch_bounds__(128) k_heavy_level(const uint32_t* __restrict__ off, uint32_t M, int S,
+__global__ void __launch_bounds__(128) k_heavy_level(const uint32_t* __restrict__ off, Group grp, int S,
                                                      uint32_t stride, const uint32_t* __restrict__ heavy,
                                                      uint32_t* __restrict__ spay) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
   if (!*heavy) return;
-  const uint32_t E = __ldg(off + M);
-  const uint32_t nchunks = (E + S - 1) / S;
+  const uint32_t G0 = __ldg(off + grp.key_lo), G1 = __ldg(off + grp.key_hi);
+  const uint32_t nchunks = (G1 - G0 + S - 1) / S;
   const uint64_t span = (uint64_t)stride * HEAVY_FAN;
   for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < nchunks; t += gridDim.x * blockDim.x) {
-    const uint32_t beg = t * (uint32_t)S;
-    const uint32_t k = find_bucket<C>(off, M, beg);
+    const uint32_t beg = G0 + t * (uint32_t)S;
+    const uint32_t k = find_bucket(off, grp.key_lo, grp.key_hi, beg);
     const uint32_t b0 = __ldg(off + k), b1 = __ldg(off + k + 1);
     if (b0 >= beg) continue;                               // chunk t has no head slot
-    const uint32_t t0 = b0 / S, t1 = (b1 - 1) / S;
+    const uint32_t t0 = (b0 - G0) / S, t1 = (b1 - 1 - G0) / S;
     if (t1 - t0 + 1 <= (uint32_t)MERGE_QMAX) continue;     // light bucket
     const uint32_t u = t - t0 - 1, nheads = t1 - t0;
     if (u % span) continue;
     typename EC_::Xyzz acc, X;
-    EC_::load(acc, spay + (size_t)(2 * t) * 4 * N);
+    EC_::load(acc, spay + (size_t)(2 * (grp.chunk_base + t)) * 4 * N);
     for (uint32_t j = 1; j < (uint32_t)HEAVY_FAN; ++j) {
       const uint64_t v = u + (uint64_t)j * stride;
       if (v >= nheads) break;
-      EC_::load(X, spay + (size_t)(2 * (t0 + 1 + v)) * 4 * N);
+      EC_::load(X, spay + (size_t)(2 * (grp.chunk_base + t0 + 1 + v)) * 4 * N);
       ec_add<C>(acc, X);
     }
-    EC_::store(spay + (size_t)(2 * t) * 4 * N, acc);
+    EC_::store(spay + (size_t)(2 * (grp.chunk_base + t)) * 4 * N, acc);
   }
 }
 
 template <class C>
-__global__ void __launch_bounds__(128) k_heavy_final(const uint32_t* __restrict__ off, uint32_t M, int S,
+__global__ void __launch_bounds__(128) k_heavy_final(const uint32_t* __restrict__ off, Group grp, int S,
                                                      const uint32_t* __restrict__ heavy,
                                                      const uint32_t* __restrict__ spay, uint32_t* __restrict__ buckets) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
   if (!*heavy) return;
-  for (uint32_t k = blockIdx.x * blockDim.x + threadIdx.x; k < M; k += gridDim.x * blockDim.x) {
+  const uint32_t G0 = __ldg(off + grp.key_lo);
+  for (uint32_t k = grp.key_lo + blockIdx.x * blockDim.x + threadIdx.x; k < grp.key_hi;
+       k += gridDim.x * blockDim.x) {
     const uint32_t b0 = __ldg(off + k), b1 = __ldg(off + k + 1);
     if (b1 == b0) continue;
-    const uint32_t t0 = b0 / S, t1 = (b1 - 1) / S;
+    const uint32_t t0 = (b0 - G0) / S, t1 = (b1 - 1 - G0) / S;
     if (t1 - t0 + 1 <= (uint32_t)MERGE_QMAX) continue;
     typename EC_::Xyzz acc, X;
-    EC_::load(acc, spay + (size_t)(2 * t0 + 1) * 4 * N);
-    EC_::load(X, spay + (size_t)(2 * (t0 + 1)) * 4 * N);
+    EC_::load(acc, spay + (size_t)(2 * (grp.chunk_base + t0) + 1) * 4 * N);
+    EC_::load(X, spay + (size_t)(2 * (grp.chunk_base + t0 + 1)) * 4 * N);
     ec_add<C>(acc, X);
     EC_::store(buckets + (size_t)k * 4 * N, acc);
   }
 }
 
 // ------------------------------------------------- a6 bucket reduction
-// Thread (t, g) owns buckets j = g*s+1 .. g*s+s of window t (digit j is stored
-// at index j-1).  Running sums from the top give R = sum_u X_u and
+// Thread (t, g) owns buckets j = g*s+1 .. g*s+s of window t_lo + t (digit j is
+// stored at index j-1).  Running sums from the top give R = sum_u X_u and
 // T = sum_u (u+1) X_u; the segment's share of W_t = sum_j j B_j is
-// T + (g s) R (PAPER.md:239's prefix-sum reduction, segmented).
+// T + (g s) R (PAPER.md:239's prefix-sum reduction, segmented).  seg_out is
+// indexed by the group-local id (t - t_lo) * G + g.
 template <class C>
 __global__ void __launch_bounds__(128) k_reduce_seg(const uint32_t* __restrict__ buckets,
-                                                    const uint32_t* __restrict__ offsets, int W, uint32_t B,
-                                                    int s, uint32_t* __restrict__ seg_out) {
+                                                    const uint32_t* __restrict__ offsets, int t_lo, int W,
+                                                    uint32_t B, int s, uint32_t* __restrict__ seg_out) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
   const uint32_t G = B / s;
   const uint32_t total = (uint32_t)W * G;
   for (uint32_t id = blockIdx.x * blockDim.x + threadIdx.x; id < total; id += gridDim.x * blockDim.x) {
-    const uint32_t t = id / G, g = id % G;
+    const uint32_t t = t_lo + id / G, g = id % G;
     typename EC_::Xyzz R, T;
     EC_::set_inf(R);
     EC_::set_inf(T);
@@ -485,24 +500,38 @@ __global__ void __launch_bounds__(128) k_reduce_win(const uint32_t* __restrict__
 
 // ----------------------------------------- a7 window combination + a8 output
 // Q = sum_t 2^(ct) W_t by Horner from the top window, on ONE warp with the
-// cooperative formulas (CoopEC).  Launch <<<1, 32>>>.  out_partial (XYZZ)
-// and/or out_affine (canonical) may be null.
+// cooperative formulas (CoopEC).  Launch <<<1, 32>>>.  The pipeline calls it
+// once per window group, top group first: windows t_hi down to t_lo; the
+// running Q is carried in `state` (XYZZ) between groups; `first` starts from
+// W_{t_hi}, `last` emits out_partial (XYZZ) and/or out_affine (canonical),
+// either of which may be null.
 template <class C>
-__global__ void __launch_bounds__(32) k_tail(const uint32_t* __restrict__ win_out, int W, int c,
+__global__ void __launch_bounds__(32) k_tail(const uint32_t* __restrict__ win_out, int t_hi, int t_lo, int c,
+                                             int first, int last, uint32_t* __restrict__ state,
                                              uint32_t* __restrict__ out_partial, uint32_t* __restrict__ out_affine) {
   using EC_ = EC<C>;
   using CO = CoopEC<C>;
   constexpr int N = C::N;
   if (blockIdx.x) return;
   typename EC_::Xyzz Q;
-  EC_::load(Q, win_out + (size_t)(W - 1) * 4 * N);
-  for (int t = W - 2; t >= 0; --t) {
+  int t = t_hi;
+  if (first) {
+    EC_::load(Q, win_out + (size_t)t * 4 * N);
+    --t;
+  } else {
+    EC_::load(Q, state);
+  }
+  for (; t >= t_lo; --t) {
     for (int k = 0; k < c; ++k) CO::dbl(Q);
     typename EC_::Xyzz X;
     EC_::load(X, win_out + (size_t)t * 4 * N);
     CO::add(Q, X);
   }
   if (threadIdx.x) return;
+  if (!last) {
+    EC_::store(state, Q);
+    return;
+  }
   if (EC_::is_inf(Q)) EC_::set_inf(Q);
   if (out_partial) EC_::store(out_partial, Q);
   if (out_affine) {
