@@ -367,7 +367,7 @@ __global__ void __launch_bounds__(128) k_merge_bucket(const uint32_t* __restrict
     EC_::load(acc, spay + (size_t)(2 * (grp.chunk_base + t0) + 1) * 4 * N);
     for (uint32_t t = t0 + 1; t <= t1; ++t) {
       EC_::load(X, spay + (size_t)(2 * (grp.chunk_base + t)) * 4 * N);
-      ec_add<C>(acc, X);
+      ec_add_hot<C>(acc, X);
     }
     EC_::store(buckets + (size_t)k * 4 * N, acc);
   }
@@ -454,12 +454,12 @@ __global__ void __launch_bounds__(128) k_reduce_seg(const uint32_t* __restrict__
       if (offsets[key + 1] != offsets[key]) {
         typename EC_::Xyzz X;
         EC_::load(X, buckets + (size_t)key * 4 * N);
-        ec_add<C>(R, X);
+        ec_add_hot<C>(R, X);
       }
-      ec_add<C>(T, R);
+      ec_add_hot<C>(T, R);
     }
-    ec_mul_small<C>(R, g * (uint32_t)s);
-    ec_add<C>(T, R);
+    ec_mul_small<C>(R, g * (uint32_t)s);      // one out-of-line call per thread
+    ec_add_hot<C>(T, R);
     EC_::store(seg_out + (size_t)id * 4 * N, T);
   }
 }
@@ -482,7 +482,7 @@ __global__ void __launch_bounds__(128) k_reduce_win(const uint32_t* __restrict__
   for (uint32_t g = lo + threadIdx.x; g < hi; g += blockDim.x) {
     typename EC_::Xyzz X;
     EC_::load(X, seg_out + ((size_t)t * G + g) * 4 * N);
-    ec_add<C>(acc, X);
+    ec_add_hot<C>(acc, X);
   }
   EC_::store(red_smem + threadIdx.x * 4 * N, acc);
   __syncthreads();
@@ -490,7 +490,7 @@ __global__ void __launch_bounds__(128) k_reduce_win(const uint32_t* __restrict__
     if (threadIdx.x < w) {
       typename EC_::Xyzz X;
       EC_::load(X, red_smem + (threadIdx.x + w) * 4 * N);
-      ec_add<C>(acc, X);
+      ec_add_hot<C>(acc, X);
       EC_::store(red_smem + threadIdx.x * 4 * N, acc);
     }
     __syncthreads();
