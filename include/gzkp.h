@@ -150,7 +150,8 @@ gzkp_status gzkp_fixed_base_mul(int curve, const void *scalars, size_t n, void *
 
 /* --- diagnostics ----------------------------------------------------------- */
 /* Elementwise field ops on canonical inputs (device arrays of n elements):
- * op 0: a*b mod p, 1: a+b, 2: a-b, 3: a^-1 (a != 0), 4: round trip to/from Montgomery. */
+ * op 0: a*b mod p, 1: a+b, 2: a-b, 3: a^-1 (a != 0), 4: round trip to/from Montgomery,
+ * 5: a^2 mod p (the dedicated Montgomery squaring). */
 gzkp_status gzkp_field_op(int curve, int op, const void *a, const void *b, void *out, size_t n,
                           gzkp_stream stream);
 /* Elementwise group ops on canonical affine points (device, n points each):

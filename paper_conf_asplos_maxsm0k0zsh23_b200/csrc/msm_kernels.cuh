@@ -643,6 +643,7 @@ __global__ void k_field_op(int op, const uint32_t* __restrict__ a, const uint32_
       case 1: Fp::add(r, x, y); break;
       case 2: Fp::sub(r, x, y); break;
       case 3: Fp::inv_canonical(r, x); break;
+      case 5: Fp::to_mont(x, x); Fp::sqr(r, x); Fp::from_mont(r, r); break;
       default: Fp::to_mont(r, x); Fp::from_mont(r, r); break;
     }
     EC_::st(out + i * N, r);
