@@ -220,7 +220,12 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    gbuild.build()
+    # the in-tree libgzkp.so travels with the repo; only a missing library is
+    # built, by rank 0 alone (never N concurrent nvcc runs)
+    if not os.path.exists(gz.LIB_PATH) and rank == 0:
+        gbuild.build()
+    if world > 1:
+        dist.barrier()
     gz.set_config(args.window_bits, args.chunk)
 
     curve, logn, cfg, sdist, desc = WORKLOADS[wl]

@@ -14,6 +14,7 @@
 // field value is canonical, so the P == Q tests are exact limb comparisons.
 #pragma once
 #include "field.cuh"
+#include "field_dfp.cuh"
 
 namespace gzkp {
 
@@ -119,6 +120,37 @@ struct EC {
     Fp::mul(t, R, t);
     Fp::mul(PPP, A.Y, PPP);
     Fp::sub(A.Y, t, PPP);               // Y3 = R(Q - X3) - Y1 PPP
+  }
+
+  // madd_nz with 4 of its 10 products on the FP64 pipe (Dfp<C>::mul, NEXT-2):
+  // one product of each dependency level that has two or more (S2, R^2, Q,
+  // Y1 PPP) goes to DFP, the rest stay on IMAD, so the two pipes work
+  // concurrently (§4.3's FP64 field arithmetic).
+  GZ_DEV static void madd_nz_mixed(Xyzz& A, const uint32_t x2[N], const uint32_t y2[N]) {
+    using D = Dfp<C>;
+    uint32_t P[N], R[N], PP[N], PPP[N], t[N];
+    Fp::mul(P, x2, A.ZZ);               // U2            (IMAD)
+    D::mul(R, y2, A.ZZZ);               // S2            (FP64)
+    Fp::sub(P, P, A.X);
+    Fp::sub(R, R, A.Y);
+    if (Fp::is_zero(P)) {
+      if (Fp::is_zero(R)) mdbl(A, x2, y2);
+      else set_inf(A);
+      return;
+    }
+    Fp::sqr(PP, P);                     // PP            (IMAD)
+    D::mul(t, R, R);                    // R^2           (FP64)
+    Fp::mul(PPP, P, PP);                // PPP           (IMAD)
+    D::mul(P, A.X, PP);                 // Q = X1 PP     (FP64)
+    Fp::mul(A.ZZ, A.ZZ, PP);            // ZZ3           (IMAD)
+    Fp::mul(A.ZZZ, A.ZZZ, PPP);         // ZZZ3          (IMAD)
+    D::mul(PP, A.Y, PPP);               // Y1 PPP        (FP64)
+    Fp::sub(t, t, PPP);
+    Fp::sub(t, t, P);
+    Fp::sub(A.X, t, P);                 // X3 = R^2 - PPP - 2Q
+    Fp::sub(t, P, A.X);
+    Fp::mul(t, R, t);                   // R (Q - X3)    (IMAD)
+    Fp::sub(A.Y, t, PP);                // Y3 = R(Q - X3) - Y1 PPP
   }
 
   // acc += B (add-2008-s), all cases.

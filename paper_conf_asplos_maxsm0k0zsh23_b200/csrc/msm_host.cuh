@@ -277,10 +277,26 @@ struct Impl {
       ss = ctx->side;
     }
     const int threads = 128;
-    const size_t acc_smem = (size_t)threads * Stage<C>::SLOT_WORDS * 4;
+    // accumulation CTA size: small CTAs let the register file hold more warps
+    // per SM (at ~176 regs/thread, 64-thread CTAs fit 10 warps, 128-thread 8)
+    static const int acc_threads = [] {
+      const char* e = getenv("GZKP_ACCUM_THREADS");
+      const int v = e ? atoi(e) : AccumCfg<C>::THREADS;
+      return (v >= 32 && v <= 128 && v % 32 == 0) ? v : AccumCfg<C>::THREADS;
+    }();
+    const size_t acc_smem = (size_t)acc_threads * Stage<C>::SLOT_WORDS * 4;
+    // NEXT-2: the hot loop with 4 of 10 products on the FP64 pipe (BLS12-381)
+    static const bool mixed = [] {
+      const char* e = getenv("GZKP_DFP");
+      return AccumCfg<C>::DFP && (e ? atoi(e) != 0 : AccumCfg<C>::DFP_DEFAULT);
+    }();
     static bool attr_set = false;
     if (!attr_set) {
-      GZ_CHECK(cudaFuncSetAttribute(k_accum<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)acc_smem));
+      GZ_CHECK(cudaFuncSetAttribute(k_accum<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
+      if constexpr (AccumCfg<C>::DFP)
+        GZ_CHECK(cudaFuncSetAttribute(k_accum<C, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
       GZ_CHECK(cudaFuncSetAttribute(k_reduce_win<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)((size_t)threads * 4 * N * 4)));
       attr_set = true;
@@ -291,8 +307,18 @@ struct Impl {
       const Group grp{gr.key_lo, gr.key_hi, (uint32_t)gr.chunk_base};
       // a4 (main stream)
       cudaEvent_t a0 = profile_event(prof, s);
-      k_accum<C><<<(unsigned)((gr.chunks_max + threads - 1) / threads), threads, acc_smem, s>>>(
-          U(p.o_vals), U(p.o_offsets), grp, pts, p.S, U(p.o_buckets), U(p.o_spay));
+      const unsigned acc_grid = (unsigned)((gr.chunks_max + acc_threads - 1) / acc_threads);
+      if constexpr (AccumCfg<C>::DFP) {
+        if (mixed)
+          k_accum<C, true><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
+                                                                   U(p.o_buckets), U(p.o_spay));
+        else
+          k_accum<C><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
+                                                             U(p.o_buckets), U(p.o_spay));
+      } else {
+        k_accum<C><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
+                                                           U(p.o_buckets), U(p.o_spay));
+      }
       GZ_CHECK(cudaGetLastError());
       cudaEvent_t a1 = profile_event(prof, s);
       profile_interval(prof, 1, a0, a1);

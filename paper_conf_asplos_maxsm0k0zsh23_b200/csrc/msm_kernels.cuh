@@ -271,13 +271,17 @@ GZ_DEV uint32_t find_bucket(const uint32_t* __restrict__ off, uint32_t lo, uint3
 template <class C>
 struct AccumCfg {
   static constexpr int MIN_CTAS = C::N <= 8 ? 3 : 1;
+  static constexpr int THREADS = 128;     // launch size (<= 128), GZKP_ACCUM_THREADS overrides
+  // FP64 (DFP) products available: 48-bit limbs tile the radix and L = 8
+  static constexpr bool DFP = C::HAS_DFP && (2 * C::N / 3 == 8);
+  static constexpr bool DFP_DEFAULT = false;   // GZKP_DFP=1 selects the mixed hot loop
 };
 
 // One chunk per thread, non-persistent grid sized for the group's worst case
 // (threads past the group's real chunk count exit): while the next group
 // accumulates, finishing CTAs free slots for the high-priority side stream
 // that merges / reduces / combines the previous group.
-template <class C>
+template <class C, bool MIXED = false>
 __global__ void __launch_bounds__(128, AccumCfg<C>::MIN_CTAS)
     k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off, Group grp,
             const uint32_t* __restrict__ pts, int S, uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay) {
@@ -336,7 +340,8 @@ __global__ void __launch_bounds__(128, AccumCfg<C>::MIN_CTAS)
       EC_::from_affine(acc, x, y);
       acc_inf = false;
     } else {
-      EC_::madd_nz(acc, x, y);
+      if constexpr (MIXED) EC_::madd_nz_mixed(acc, x, y);   // IMAD + FP64 pipes (NEXT-2)
+      else EC_::madd_nz(acc, x, y);
       acc_inf = EC_::is_inf(acc);
     }
   }
@@ -644,6 +649,11 @@ __global__ void k_field_op(int op, const uint32_t* __restrict__ a, const uint32_
       case 2: Fp::sub(r, x, y); break;
       case 3: Fp::inv_canonical(r, x); break;
       case 5: Fp::to_mont(x, x); Fp::sqr(r, x); Fp::from_mont(r, r); break;
+      case 6:   // FP64 (DFP) Montgomery product where available, else the IMAD one
+        Fp::to_mont(x, x); Fp::to_mont(y, y);
+        if constexpr (AccumCfg<C>::DFP) Dfp<C>::mul(r, x, y); else Fp::mul(r, x, y);
+        Fp::from_mont(r, r);
+        break;
       default: Fp::to_mont(r, x); Fp::from_mont(r, r); break;
     }
     EC_::st(out + i * N, r);
