@@ -324,16 +324,47 @@ gzkp_status gzkp_msm_host(int curve, const void* points_host, const void* scalar
   init_pool_once();
   cudaStream_t s = (cudaStream_t)stream;
   const size_t pb = n * 2 * c->limbs * 4, sb = n * c->scalar_limbs * 4, ob = 2 * c->limbs * 4;
+  // staging (canonical points as copied), Montgomery points, scalars, out
   char* d = nullptr;
-  const size_t total = align_up(pb) + align_up(sb) + align_up(ob);
+  const size_t total = 2 * align_up(pb) + align_up(sb) + align_up(ob);
   cudaError_t e = cudaMallocAsync((void**)&d, total, s);
   if (e != cudaSuccess) return cuda_status(e, "cudaMallocAsync");
-  void *dp = d, *ds = d + align_up(pb), *dout = d + align_up(pb) + align_up(sb);
+  char *dstage = d, *dp = d + align_up(pb), *ds = d + 2 * align_up(pb), *dout = ds + align_up(sb);
   gzkp_status st = GZKP_SUCCESS;
-  if (n && (e = cudaMemcpyAsync(dp, points_host, pb, cudaMemcpyHostToDevice, s)) != cudaSuccess) st = cuda_status(e, "H2D points");
-  if (!st && n && (e = cudaMemcpyAsync(ds, scalars_host, sb, cudaMemcpyHostToDevice, s)) != cudaSuccess) st = cuda_status(e, "H2D scalars");
-  if (!st) st = gzkp_msm(curve, dp, ds, n, dout, stream);
+  StreamCtx* ctx = nullptr;
+  if ((st = stream_ctx(s, &ctx))) { cudaFreeAsync(d, s); return st; }
+  cudaStream_t ss = ctx->side;
+  cudaEvent_t ev_alloc = ctx->ev[ctx->nev - 3], ev_points = ctx->ev[ctx->nev - 2];
+  // points on the side stream, in chunks, each converted to Montgomery form as
+  // it lands; the scalars go first on the caller's stream so the digits and
+  // the sort overlap the (larger) point transfer ("async copies")
+  if ((e = cudaEventRecord(ev_alloc, s)) != cudaSuccess || (e = cudaStreamWaitEvent(ss, ev_alloc, 0)) != cudaSuccess)
+    st = cuda_status(e, "event");
+  const size_t chunk = std::max<size_t>(1, (64u << 20) / (2 * c->limbs * 4));
+  for (size_t off = 0; !st && off < n; off += chunk) {
+    const size_t cnt = std::min(chunk, n - off);
+    const size_t boff = off * 2 * c->limbs * 4;
+    if ((e = cudaMemcpyAsync(dstage + boff, (const char*)points_host + boff, cnt * 2 * c->limbs * 4,
+                             cudaMemcpyHostToDevice, ss)) != cudaSuccess)
+      st = cuda_status(e, "H2D points");
+    if (!st) st = c->to_mont(dstage + boff, dp + boff, cnt, ss);
+  }
+  if (!st && (e = cudaEventRecord(ev_points, ss)) != cudaSuccess) st = cuda_status(e, "event");
+  if (!st && n && (e = cudaMemcpyAsync(ds, scalars_host, sb, cudaMemcpyHostToDevice, s)) != cudaSuccess)
+    st = cuda_status(e, "H2D scalars");
+  if (!st) {
+    MsmCall call;
+    call.points = dp;
+    call.prepared = true;            // already Montgomery (converted per chunk above)
+    call.scalars = ds;
+    call.n = n;
+    call.out_affine = dout;
+    call.stream = s;
+    call.points_ready = n ? ev_points : nullptr;
+    st = n ? c->msm(call) : c->msm(call);
+  }
   if (!st && (e = cudaMemcpyAsync(out_host, dout, ob, cudaMemcpyDeviceToHost, s)) != cudaSuccess) st = cuda_status(e, "D2H out");
+  cudaStreamWaitEvent(s, ev_points, 0);   // never free while the side stream may still copy
   cudaFreeAsync(d, s);
   if ((e = cudaStreamSynchronize(s)) != cudaSuccess && !st) st = cuda_status(e, "cudaStreamSynchronize");
   return st;

@@ -27,6 +27,7 @@ struct MsmCall {
   bool consolidated = false;      // points = weighted-point table [W][table_n] (NEXT-1)
   int window_bits = 0;            // forced c (0 = planner); set for consolidated tables
   size_t table_n = 0;
+  cudaEvent_t points_ready = nullptr;   // if set: the accumulation waits for it (overlapped H2D)
   const void* scalars = nullptr;
   size_t n = 0;
   void* out_affine = nullptr;     // canonical affine result (may be null)

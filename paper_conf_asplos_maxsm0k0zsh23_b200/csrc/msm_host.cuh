@@ -301,6 +301,9 @@ struct Impl {
                                     (int)((size_t)threads * 4 * N * 4)));
       attr_set = true;
     }
+    // overlapped host->device path: the points are still arriving on another
+    // stream while the digits / sort ran; only the accumulation needs them
+    if (call.points_ready) GZ_CHECK(cudaStreamWaitEvent(s, call.points_ready, 0));
     cudaEvent_t ev_last_acc = nullptr, ev_merged = nullptr, ev_reduced = nullptr, ev_tailed = nullptr;
     for (int gi = 0; gi < ngroups; ++gi) {
       const auto& gr = p.groups[gi];
