@@ -152,8 +152,13 @@ struct Impl {
       const uint64_t wins = consolidated ? (uint64_t)p.W : (uint64_t)(g.t_hi - g.t_lo + 1);
       const uint64_t bwins = consolidated ? 1 : wins;
       // reduction segment of this group: <= 16 buckets, fewer until >= 32K threads
+      static const uint64_t target = [] {
+        const char* e = getenv("GZKP_REDUCE_THREADS");
+        const long v = e ? atol(e) : 32768;
+        return (uint64_t)(v > 0 ? v : 32768);
+      }();
       uint64_t seg = 16;
-      while (seg > 1 && bwins * p.B / seg < 32768) seg >>= 1;
+      while (seg > 1 && bwins * p.B / seg < target) seg >>= 1;
       g.seg = (int)std::min<uint64_t>(seg, p.B);
       const uint64_t gsegs = p.B / g.seg;
       seg_elems = std::max<uint64_t>(seg_elems, bwins * gsegs);
