@@ -53,6 +53,12 @@ def lib():
             "oracle_msm": [ctypes.c_int, u32p, u32p, u32p, u32p, ctypes.c_int, ctypes.c_uint64, u32p, ctypes.c_int],
             "oracle_mul_each": [ctypes.c_int, u32p, u32p, u32p, u32p, ctypes.c_int, ctypes.c_uint64, u32p, ctypes.c_int],
             "oracle_ec_add": [ctypes.c_int, u32p, u32p, u32p, u32p, u32p],
+            "oracle_msm_ext": [ctypes.c_int, ctypes.c_int, u32p, u32p, u32p, u32p, u32p, ctypes.c_int,
+                               ctypes.c_uint64, u32p, ctypes.c_int],
+            "oracle_mul_each_ext": [ctypes.c_int, ctypes.c_int, u32p, u32p, u32p, u32p, u32p, ctypes.c_int,
+                                    ctypes.c_uint64, u32p, ctypes.c_int],
+            "oracle_ec_add_ext": [ctypes.c_int, ctypes.c_int, u32p, u32p, u32p, u32p, u32p, u32p],
+            "oracle_fp2_mul": [ctypes.c_int, u32p, u32p, u32p, u32p, u32p],
             "oracle_fp_mul": [ctypes.c_int, u32p, u32p, u32p, u32p],
             "oracle_fp_inv": [ctypes.c_int, u32p, u32p, u32p],
             "oracle_bn_mod": [u32p, ctypes.c_int, u32p, ctypes.c_int, u32p],
@@ -80,40 +86,50 @@ def _u32(a) -> np.ndarray:
 
 
 def _consts(c: Curve):
+    """(L, deg, p, beta, a) limb arrays for the C oracle."""
     L = c.limbs
-    return L, _u32(ref.int_to_limbs(c.p, L)), _u32(ref.int_to_limbs(c.a % c.p, L))
+    if c.deg == 2:
+        a = ref.int_to_limbs(c.a[0] % c.p, L) + ref.int_to_limbs(c.a[1] % c.p, L)
+        beta = ref.int_to_limbs(c.beta % c.p, L)
+    else:
+        a = ref.int_to_limbs(c.a % c.p, L)
+        beta = [0] * L
+    return L, c.deg, _u32(ref.int_to_limbs(c.p, L)), _u32(beta), _u32(a)
 
 
 def msm(curve, points: np.ndarray, scalars: np.ndarray, nthreads: int | None = None) -> np.ndarray:
-    """C oracle MSM.  points: [n, 2L] u32 canonical affine ((0,0) = O);
-    scalars: [n, Ls] u32 little-endian.  Returns [2L] u32 (affine, (0,0) = O)."""
+    """C oracle MSM.  points: [n, 2D] u32 canonical affine ((0,0) = O; D =
+    deg * L limbs per coordinate); scalars: [n, Ls] u32 little-endian.
+    Returns [2D] u32 (affine, (0,0) = O)."""
     c = get(curve)
-    L, p, a = _consts(c)
-    points = _u32(points).reshape(-1, 2 * L)
+    L, deg, p, beta, a = _consts(c)
+    D = deg * L
+    points = _u32(points).reshape(-1, 2 * D)
     scalars = _u32(scalars)
     n = points.shape[0]
     Ls = scalars.shape[1] if scalars.ndim == 2 else 1
     scalars = scalars.reshape(n, Ls)
-    out = np.zeros(2 * L, dtype=np.uint32)
-    rc = lib().oracle_msm(L, _p(p), _p(a), _p(points), _p(scalars), Ls, n, _p(out),
-                          nthreads or default_threads())
+    out = np.zeros(2 * D, dtype=np.uint32)
+    rc = lib().oracle_msm_ext(L, deg, _p(p), _p(beta), _p(a), _p(points), _p(scalars), Ls, n, _p(out),
+                              nthreads or default_threads())
     if rc:
         raise RuntimeError(f"oracle_msm failed: {rc}")
     return out
 
 
 def mul_each(curve, P: np.ndarray, scalars: np.ndarray, nthreads: int | None = None) -> np.ndarray:
-    """out[i] = k_i (x) P (C oracle).  Returns [n, 2L] u32."""
+    """out[i] = k_i (x) P (C oracle).  Returns [n, 2D] u32."""
     c = get(curve)
-    L, p, a = _consts(c)
-    P = _u32(P).reshape(2 * L)
+    L, deg, p, beta, a = _consts(c)
+    D = deg * L
+    P = _u32(P).reshape(2 * D)
     scalars = _u32(scalars)
     n = scalars.shape[0]
     Ls = scalars.shape[1] if scalars.ndim == 2 else 1
     scalars = scalars.reshape(n, Ls)
-    out = np.zeros((n, 2 * L), dtype=np.uint32)
-    rc = lib().oracle_mul_each(L, _p(p), _p(a), _p(P), _p(scalars), Ls, n, _p(out),
-                               nthreads or default_threads())
+    out = np.zeros((n, 2 * D), dtype=np.uint32)
+    rc = lib().oracle_mul_each_ext(L, deg, _p(p), _p(beta), _p(a), _p(P), _p(scalars), Ls, n, _p(out),
+                                   nthreads or default_threads())
     if rc:
         raise RuntimeError(f"oracle_mul_each failed: {rc}")
     return out
@@ -132,9 +148,9 @@ def points_from_dlogs(curve, dlogs: np.ndarray, nthreads: int | None = None) -> 
 
 def ec_add(curve, P: np.ndarray, Q: np.ndarray) -> np.ndarray:
     c = get(curve)
-    L, p, a = _consts(c)
-    out = np.zeros(2 * L, dtype=np.uint32)
-    rc = lib().oracle_ec_add(L, _p(p), _p(a), _p(_u32(P)), _p(_u32(Q)), _p(out))
+    L, deg, p, beta, a = _consts(c)
+    out = np.zeros(2 * deg * L, dtype=np.uint32)
+    rc = lib().oracle_ec_add_ext(L, deg, _p(p), _p(beta), _p(a), _p(_u32(P)), _p(_u32(Q)), _p(out))
     if rc:
         raise RuntimeError(f"oracle_ec_add failed: {rc}")
     return out
@@ -142,7 +158,8 @@ def ec_add(curve, P: np.ndarray, Q: np.ndarray) -> np.ndarray:
 
 def fp_mul(curve, x: int, y: int) -> int:
     c = get(curve)
-    L, p, _ = _consts(c)
+    L = c.limbs
+    p = _u32(ref.int_to_limbs(c.p, L))
     out = np.zeros(L, dtype=np.uint32)
     X, Y = _u32(ref.int_to_limbs(x, L)), _u32(ref.int_to_limbs(y, L))
     if lib().oracle_fp_mul(L, _p(p), _p(X), _p(Y), _p(out)):
@@ -150,9 +167,22 @@ def fp_mul(curve, x: int, y: int) -> int:
     return ref.limbs_to_int(out)
 
 
+def fp2_mul(curve, x, y):
+    """x * y in the G2 curve's F_p^2 (C oracle); x, y = (c0, c1)."""
+    c = get(curve)
+    L, _, p, beta, _ = _consts(c)
+    X = _u32(ref.int_to_limbs(x[0], L) + ref.int_to_limbs(x[1], L))
+    Y = _u32(ref.int_to_limbs(y[0], L) + ref.int_to_limbs(y[1], L))
+    out = np.zeros(2 * L, dtype=np.uint32)
+    if lib().oracle_fp2_mul(L, _p(p), _p(beta), _p(X), _p(Y), _p(out)):
+        raise RuntimeError("oracle_fp2_mul failed")
+    return (ref.limbs_to_int(out[:L]), ref.limbs_to_int(out[L:]))
+
+
 def fp_inv(curve, x: int) -> int:
     c = get(curve)
-    L, p, _ = _consts(c)
+    L = c.limbs
+    p = _u32(ref.int_to_limbs(c.p, L))
     out = np.zeros(L, dtype=np.uint32)
     X = _u32(ref.int_to_limbs(x, L))
     if lib().oracle_fp_inv(L, _p(p), _p(X), _p(out)):
@@ -202,4 +232,4 @@ def dot_mod(scalars: np.ndarray, dlogs: np.ndarray, r: int) -> int:
 
 
 __all__ = ["curves", "ref", "msm", "mul_each", "points_from_dlogs", "closed_form", "dot_mod",
-           "ec_add", "fp_mul", "fp_inv", "bn_mod", "build", "default_threads", "generator_limbs"]
+           "ec_add", "fp_mul", "fp2_mul", "fp_inv", "bn_mod", "build", "default_threads", "generator_limbs"]

@@ -25,12 +25,19 @@ class Curve:
     cid: int          # id shared with the C ABI enum (gzkp_curve)
     p: int            # base field modulus q (PAPER.md:106 calls it F_q)
     r: int            # order of the G1 group = scalar field modulus (PAPER.md:105 F_r)
-    a: int
-    b: int
-    gx: int
-    gy: int
-    cofactor: int     # #E(F_p) / r
+    a: object         # int for G1; (c0, c1) in F_p^2 for G2
+    b: object
+    gx: object
+    gy: object
+    cofactor: int     # #E(F_p) / r   (G2: #E'(F_p^2) / r)
     scalar_bits: int  # b = bit length of r: scalars are integers < 2^scalar_bits
+    deg: int = 1      # 1: G1 over F_p; 2: G2 over F_p^2 = F_p[u]/(u^2 - beta)
+    beta: int = 0     # deg 2 only
+
+    @property
+    def coord_limbs(self) -> int:
+        """u32 limbs of one curve coordinate (deg F_p coordinates c0 || c1)."""
+        return self.deg * self.limbs
 
     @property
     def limbs(self) -> int:
@@ -104,7 +111,35 @@ def _toy_generator(c: Curve) -> Curve:
 TOY_A0 = _toy_generator(TOY_A0)
 TOY_A2 = _toy_generator(TOY_A2)
 
-CURVES = {c.name: c for c in (BN254, BLS12_381, MNT4_753, TOY_A0, TOY_A2)}
+# ---- G2 (GZKP's MSM optimisations "apply to both G1 and G2";
+# Groth16's B-query lives in G2).  G2 is the order-r subgroup of a sextic twist
+# E'(F_p^2): y^2 = x^3 + b' over F_p^2 = F_p[u]/(u^2 + 1) (DESIGN.md reading
+# R14).  b' and the generators are the standard published values (EIP-197 for
+# BN254; the IETF pairing-friendly-curves draft / zkcrypto for BLS12-381);
+# tests/test_oracle_pins.py pins them: b'(9 + u) = 3 resp. b' = 4(1 + u),
+# G2 on E', r G2 = O, G2 != O.
+BN254_G2 = Curve(
+    name="bn254_g2", cid=3, p=BN254.p, r=BN254.r, a=(0, 0),
+    b=(_h("2b149d40ceb8aaae81be18991be06ac3b5b4c5e559dbefa33267e6dc24a138e5"),
+       _h("009713b03af0fed4cd2cafadeed8fdf4a74fa084e52d1852e4a2bd0685c315d2")),
+    gx=(10857046999023057135944570762232829481370756359578518086990519993285655852781,
+        11559732032986387107991004021392285783925812861821192530917403151452391805634),
+    gy=(8495653923123431417604973247489272438418190587263600148770280649306958101930,
+        4082367875863433681332203403145435568316851327593401208105741076214120093531),
+    cofactor=2 * BN254.p - BN254.r, scalar_bits=254, deg=2, beta=BN254.p - 1,
+)
+
+BLS12_381_G2 = Curve(
+    name="bls12_381_g2", cid=4, p=BLS12_381.p, r=BLS12_381.r, a=(0, 0), b=(4, 4),
+    gx=(_h("024aa2b2f08f0a91260805272dc51051c6e47ad4fa403b02b4510b647ae3d1770bac0326a805bbefd48056c8c121bdb8"),
+        _h("13e02b6052719f607dacd3a088274f65596bd0d09920b61ab5da61bbdc7f5049334cf11213945d57e5ac7d055d042b7e")),
+    gy=(_h("0ce5d527727d6e118cc9cdc6da2e351aadfd9baa8cbdd3a76d429a695160d12c923ac9cc3baca289e193548608b82801"),
+        _h("0606c4a02ea734cc32acd2b02bc28b99cb3e287e85a763af267492ab572e99ab3f370d275cec1da1aaa9075ff05f79be")),
+    cofactor=_h("5d543a95414e7f1091d50792876a202cd91de4547085abaa68a205b2e5a7ddfa628f1cb4d9e82ef21537e293a6691ae1616ec6e786f0c70cf1c38e31c7238e5"),
+    scalar_bits=255, deg=2, beta=BLS12_381.p - 1,
+)
+
+CURVES = {c.name: c for c in (BN254, BLS12_381, MNT4_753, TOY_A0, TOY_A2, BN254_G2, BLS12_381_G2)}
 BY_ID = {c.cid: c for c in CURVES.values()}
 
 

@@ -22,9 +22,15 @@
  *      are added in chunk order.  The group is abelian and exact, so the
  *      result is independent of the order.
  *
- * Encoding: a point is 2L little-endian u32 limbs x || y, canonical (< p);
- * the identity O is (0,0).  A scalar is Ls little-endian u32 limbs, any
- * integer (not reduced mod r).
+ * G2 (the MSM optimisations "apply to both G1 and G2") is the
+ * same definition over F_p^2 = F_p[u]/(u^2 - beta): an element is c0 + c1 u,
+ * stored c0 || c1, and its product is the schoolbook polynomial product
+ * reduced by u^2 = beta (no Karatsuba: plain definition).
+ *
+ * Encoding: a point is 2D little-endian u32 limbs x || y (D = deg * L limbs
+ * per coordinate), canonical (< p per F_p coordinate); the identity O is
+ * (0,0).  A scalar is Ls little-endian u32 limbs, any integer (not reduced
+ * mod r).
  */
 #include <pthread.h>
 #include <stdint.h>
@@ -34,14 +40,17 @@
 #define MAXL 24
 
 typedef struct {
-    int L;               /* limbs of the encoding */
+    int L;               /* limbs of one F_p coordinate in the encoding */
     int Le;              /* effective limbs of p (top limb nonzero) */
+    int deg;             /* 1: E(F_p) (G1); 2: E'(F_p^2) (G2, the twist) */
+    int D;               /* limbs of one curve coordinate = deg * L */
     uint32_t p[MAXL];
-    uint32_t a[MAXL];
+    uint32_t beta[MAXL]; /* deg 2: F_p^2 = F_p[u] / (u^2 - beta) */
+    uint32_t a[2 * MAXL];/* curve coefficient a, deg coordinates */
 } fctx;
 
 typedef struct {
-    uint32_t x[MAXL], y[MAXL];
+    uint32_t x[2 * MAXL], y[2 * MAXL];
     int inf;             /* 1 = identity O */
 } apt;
 
@@ -217,43 +226,88 @@ static void fp_inv(const fctx *f, uint32_t *r, const uint32_t *x) {
     memcpy(r, bn_is_one(u, L) ? x1 : x2, sizeof(uint32_t) * L);
 }
 
+/* --------------------------------------------- F_p^deg (deg = 1 or 2) */
+/* An element is deg F_p coordinates; for deg 2, c0 + c1 u with u^2 = beta. */
+
+static void fe_add(const fctx *f, uint32_t *r, const uint32_t *x, const uint32_t *y) {
+    for (int i = 0; i < f->deg; ++i) fp_add(f, r + i * f->L, x + i * f->L, y + i * f->L);
+}
+
+static void fe_sub(const fctx *f, uint32_t *r, const uint32_t *x, const uint32_t *y) {
+    for (int i = 0; i < f->deg; ++i) fp_sub(f, r + i * f->L, x + i * f->L, y + i * f->L);
+}
+
+/* (x0 + x1 u)(y0 + y1 u) = (x0 y0 + beta x1 y1) + (x0 y1 + x1 y0) u */
+static void fe_mul(const fctx *f, uint32_t *r, const uint32_t *x, const uint32_t *y) {
+    if (f->deg == 1) { fp_mul(f, r, x, y); return; }
+    int L = f->L;
+    uint32_t t0[MAXL], t1[MAXL], t2[MAXL], r0[MAXL], r1[MAXL];
+    fp_mul(f, t0, x, y);                 /* x0 y0 */
+    fp_mul(f, t1, x + L, y + L);         /* x1 y1 */
+    fp_mul(f, t2, f->beta, t1);          /* beta x1 y1 */
+    fp_add(f, r0, t0, t2);
+    fp_mul(f, t0, x, y + L);             /* x0 y1 */
+    fp_mul(f, t1, x + L, y);             /* x1 y0 */
+    fp_add(f, r1, t0, t1);
+    memcpy(r, r0, sizeof(uint32_t) * L);
+    memcpy(r + L, r1, sizeof(uint32_t) * L);
+}
+
+/* 1 / (x0 + x1 u) = (x0 - x1 u) / (x0^2 - beta x1^2); x != 0 required */
+static void fe_inv(const fctx *f, uint32_t *r, const uint32_t *x) {
+    if (f->deg == 1) { fp_inv(f, r, x); return; }
+    int L = f->L;
+    uint32_t t0[MAXL], t1[MAXL], nrm[MAXL], ni[MAXL], zero[MAXL];
+    memset(zero, 0, sizeof(zero));
+    fp_mul(f, t0, x, x);
+    fp_mul(f, t1, x + L, x + L);
+    fp_mul(f, t1, f->beta, t1);
+    fp_sub(f, nrm, t0, t1);              /* the norm, in F_p */
+    fp_inv(f, ni, nrm);
+    fp_mul(f, t0, x, ni);
+    fp_sub(f, t1, zero, x + L);
+    fp_mul(f, t1, t1, ni);
+    memcpy(r, t0, sizeof(uint32_t) * L);
+    memcpy(r + L, t1, sizeof(uint32_t) * L);
+}
+
 /* ------------------------------------------------------------ group law */
 
 static void ec_add(const fctx *f, apt *R, const apt *P, const apt *Q) {
-    int L = f->L;
+    int D = f->D;
     if (P->inf) { *R = *Q; return; }
     if (Q->inf) { *R = *P; return; }
-    uint32_t lam[MAXL], num[MAXL], den[MAXL], t[MAXL];
-    if (bn_cmp(P->x, Q->x, L) == 0) {
-        fp_add(f, t, P->y, Q->y);
-        if (bn_is_zero(t, L)) {             /* P == -Q */
+    uint32_t lam[2 * MAXL], num[2 * MAXL], den[2 * MAXL], t[2 * MAXL];
+    if (bn_cmp(P->x, Q->x, D) == 0) {
+        fe_add(f, t, P->y, Q->y);
+        if (bn_is_zero(t, D)) {             /* P == -Q */
             memset(R, 0, sizeof(*R));
             R->inf = 1;
             return;
         }
         /* tangent: lam = (3 x^2 + a) / (2 y) */
-        fp_mul(f, t, P->x, P->x);
-        fp_add(f, num, t, t);
-        fp_add(f, num, num, t);
-        fp_add(f, num, num, f->a);
-        fp_add(f, den, P->y, P->y);
+        fe_mul(f, t, P->x, P->x);
+        fe_add(f, num, t, t);
+        fe_add(f, num, num, t);
+        fe_add(f, num, num, f->a);
+        fe_add(f, den, P->y, P->y);
     } else {
         /* chord: lam = (y2 - y1) / (x2 - x1) */
-        fp_sub(f, num, Q->y, P->y);
-        fp_sub(f, den, Q->x, P->x);
+        fe_sub(f, num, Q->y, P->y);
+        fe_sub(f, den, Q->x, P->x);
     }
-    fp_inv(f, t, den);
-    fp_mul(f, lam, num, t);
-    uint32_t x3[MAXL], y3[MAXL];
-    fp_mul(f, x3, lam, lam);
-    fp_sub(f, x3, x3, P->x);
-    fp_sub(f, x3, x3, Q->x);
-    fp_sub(f, t, P->x, x3);
-    fp_mul(f, y3, lam, t);
-    fp_sub(f, y3, y3, P->y);
+    fe_inv(f, t, den);
+    fe_mul(f, lam, num, t);
+    uint32_t x3[2 * MAXL], y3[2 * MAXL];
+    fe_mul(f, x3, lam, lam);
+    fe_sub(f, x3, x3, P->x);
+    fe_sub(f, x3, x3, Q->x);
+    fe_sub(f, t, P->x, x3);
+    fe_mul(f, y3, lam, t);
+    fe_sub(f, y3, y3, P->y);
     memset(R, 0, sizeof(*R));
-    memcpy(R->x, x3, sizeof(uint32_t) * L);
-    memcpy(R->y, y3, sizeof(uint32_t) * L);
+    memcpy(R->x, x3, sizeof(uint32_t) * D);
+    memcpy(R->y, y3, sizeof(uint32_t) * D);
     R->inf = 0;
 }
 
@@ -276,26 +330,30 @@ static void ec_mul(const fctx *f, apt *R, const uint32_t *k, int Ls, const apt *
 
 static void load_point(const fctx *f, apt *P, const uint32_t *src) {
     memset(P, 0, sizeof(*P));
-    memcpy(P->x, src, sizeof(uint32_t) * f->L);
-    memcpy(P->y, src + f->L, sizeof(uint32_t) * f->L);
-    P->inf = bn_is_zero(P->x, f->L) && bn_is_zero(P->y, f->L);
+    memcpy(P->x, src, sizeof(uint32_t) * f->D);
+    memcpy(P->y, src + f->D, sizeof(uint32_t) * f->D);
+    P->inf = bn_is_zero(P->x, f->D) && bn_is_zero(P->y, f->D);
 }
 
 static void store_point(const fctx *f, uint32_t *dst, const apt *P) {
     if (P->inf) {
-        memset(dst, 0, sizeof(uint32_t) * 2 * f->L);
+        memset(dst, 0, sizeof(uint32_t) * 2 * f->D);
         return;
     }
-    memcpy(dst, P->x, sizeof(uint32_t) * f->L);
-    memcpy(dst + f->L, P->y, sizeof(uint32_t) * f->L);
+    memcpy(dst, P->x, sizeof(uint32_t) * f->D);
+    memcpy(dst + f->D, P->y, sizeof(uint32_t) * f->D);
 }
 
-static int init_ctx(fctx *f, int L, const uint32_t *p, const uint32_t *a) {
-    if (L < 1 || L > MAXL) return -1;
+/* deg 1: beta unused (may be NULL); a has deg * L limbs */
+static int init_ctx(fctx *f, int L, int deg, const uint32_t *p, const uint32_t *beta, const uint32_t *a) {
+    if (L < 1 || L > MAXL || (deg != 1 && deg != 2)) return -1;
     memset(f, 0, sizeof(*f));
     f->L = L;
+    f->deg = deg;
+    f->D = deg * L;
     memcpy(f->p, p, sizeof(uint32_t) * L);
-    memcpy(f->a, a, sizeof(uint32_t) * L);
+    if (deg == 2) memcpy(f->beta, beta, sizeof(uint32_t) * L);
+    memcpy(f->a, a, sizeof(uint32_t) * f->D);
     f->Le = L;
     while (f->Le > 1 && f->p[f->Le - 1] == 0) f->Le--;
     if (!(f->p[0] & 1)) return -1;
@@ -322,7 +380,7 @@ static void *run_job(void *arg) {
     for (uint64_t i = j->begin; i < j->end; ++i) {
         apt P, R;
         const uint32_t *k = j->scalars + (size_t)i * j->Ls;
-        load_point(f, &P, j->points + (j->each ? 0 : (size_t)i * 2 * f->L));
+        load_point(f, &P, j->points + (j->each ? 0 : (size_t)i * 2 * f->D));
         if (P.inf || bn_is_zero(k, j->Ls)) {
             memset(&R, 0, sizeof(R));
             R.inf = 1;
@@ -330,7 +388,7 @@ static void *run_job(void *arg) {
             ec_mul(f, &R, k, j->Ls, &P);
         }
         if (j->each) {
-            store_point(f, j->out + (size_t)i * 2 * f->L, &R);
+            store_point(f, j->out + (size_t)i * 2 * f->D, &R);
         } else {
             apt t;
             ec_add(f, &t, &acc, &R);
@@ -347,7 +405,7 @@ static int run_parallel(const fctx *f, const uint32_t *points, const uint32_t *s
     if ((uint64_t)nthreads > n) nthreads = n ? (int)n : 1;
     job *jobs = (job *)calloc(nthreads, sizeof(job));
     pthread_t *th = (pthread_t *)calloc(nthreads, sizeof(pthread_t));
-    uint32_t *partial = (uint32_t *)calloc((size_t)nthreads * 2 * f->L, sizeof(uint32_t));
+    uint32_t *partial = (uint32_t *)calloc((size_t)nthreads * 2 * f->D, sizeof(uint32_t));
     if (!jobs || !th || !partial) { free(jobs); free(th); free(partial); return -2; }
     uint64_t chunk = (n + nthreads - 1) / nthreads;
     for (int t = 0; t < nthreads; ++t) {
@@ -357,7 +415,7 @@ static int run_parallel(const fctx *f, const uint32_t *points, const uint32_t *s
         jobs[t].Ls = Ls;
         jobs[t].begin = (uint64_t)t * chunk < n ? (uint64_t)t * chunk : n;
         jobs[t].end = (uint64_t)(t + 1) * chunk < n ? (uint64_t)(t + 1) * chunk : n;
-        jobs[t].out = each ? out : partial + (size_t)t * 2 * f->L;
+        jobs[t].out = each ? out : partial + (size_t)t * 2 * f->D;
         jobs[t].each = each;
         pthread_create(&th[t], NULL, run_job, &jobs[t]);
     }
@@ -367,7 +425,7 @@ static int run_parallel(const fctx *f, const uint32_t *points, const uint32_t *s
         memset(&acc, 0, sizeof(acc));
         acc.inf = 1;
         for (int t = 0; t < nthreads; ++t) {
-            load_point(f, &P, partial + (size_t)t * 2 * f->L);
+            load_point(f, &P, partial + (size_t)t * 2 * f->D);
             ec_add(f, &s, &acc, &P);
             acc = s;
         }
@@ -381,27 +439,30 @@ static int run_parallel(const fctx *f, const uint32_t *points, const uint32_t *s
 
 /* ------------------------------------------------------------- exports */
 
-/* Q = sum k_i P_i.  points: n x 2L limbs; scalars: n x Ls limbs; out: 2L limbs. */
-int oracle_msm(int L, const uint32_t *p, const uint32_t *a, const uint32_t *points,
-               const uint32_t *scalars, int Ls, uint64_t n, uint32_t *out, int nthreads) {
+/* Q = sum k_i P_i over E(F_p^deg).  points: n x 2 deg L limbs; scalars: n x Ls
+ * limbs; out: 2 deg L limbs.  beta: deg 2 only (u^2 = beta); a: deg L limbs. */
+int oracle_msm_ext(int L, int deg, const uint32_t *p, const uint32_t *beta, const uint32_t *a,
+                   const uint32_t *points, const uint32_t *scalars, int Ls, uint64_t n, uint32_t *out,
+                   int nthreads) {
     fctx f;
-    if (init_ctx(&f, L, p, a)) return -1;
+    if (init_ctx(&f, L, deg, p, beta, a)) return -1;
     return run_parallel(&f, points, scalars, Ls, n, out, nthreads, 0);
 }
 
-/* out_i = k_i P for one base point P (2L limbs); out: n x 2L limbs. */
-int oracle_mul_each(int L, const uint32_t *p, const uint32_t *a, const uint32_t *P,
-                    const uint32_t *scalars, int Ls, uint64_t n, uint32_t *out, int nthreads) {
+/* out_i = k_i P for one base point P; out: n points. */
+int oracle_mul_each_ext(int L, int deg, const uint32_t *p, const uint32_t *beta, const uint32_t *a,
+                        const uint32_t *P, const uint32_t *scalars, int Ls, uint64_t n, uint32_t *out,
+                        int nthreads) {
     fctx f;
-    if (init_ctx(&f, L, p, a)) return -1;
+    if (init_ctx(&f, L, deg, p, beta, a)) return -1;
     return run_parallel(&f, P, scalars, Ls, n, out, nthreads, 1);
 }
 
 /* R = P + Q (affine, explicit cases) */
-int oracle_ec_add(int L, const uint32_t *p, const uint32_t *a, const uint32_t *P,
-                  const uint32_t *Q, uint32_t *R) {
+int oracle_ec_add_ext(int L, int deg, const uint32_t *p, const uint32_t *beta, const uint32_t *a,
+                      const uint32_t *P, const uint32_t *Q, uint32_t *R) {
     fctx f;
-    if (init_ctx(&f, L, p, a)) return -1;
+    if (init_ctx(&f, L, deg, p, beta, a)) return -1;
     apt A, B, C;
     load_point(&f, &A, P);
     load_point(&f, &B, Q);
@@ -410,10 +471,36 @@ int oracle_ec_add(int L, const uint32_t *p, const uint32_t *a, const uint32_t *P
     return 0;
 }
 
+/* G1 forms (deg 1) */
+int oracle_msm(int L, const uint32_t *p, const uint32_t *a, const uint32_t *points,
+               const uint32_t *scalars, int Ls, uint64_t n, uint32_t *out, int nthreads) {
+    return oracle_msm_ext(L, 1, p, NULL, a, points, scalars, Ls, n, out, nthreads);
+}
+
+int oracle_mul_each(int L, const uint32_t *p, const uint32_t *a, const uint32_t *P,
+                    const uint32_t *scalars, int Ls, uint64_t n, uint32_t *out, int nthreads) {
+    return oracle_mul_each_ext(L, 1, p, NULL, a, P, scalars, Ls, n, out, nthreads);
+}
+
+int oracle_ec_add(int L, const uint32_t *p, const uint32_t *a, const uint32_t *P,
+                  const uint32_t *Q, uint32_t *R) {
+    return oracle_ec_add_ext(L, 1, p, NULL, a, P, Q, R);
+}
+
+/* r = x * y in F_p^2 (u^2 = beta), exported for the field pins */
+int oracle_fp2_mul(int L, const uint32_t *p, const uint32_t *beta, const uint32_t *x, const uint32_t *y,
+                   uint32_t *r) {
+    fctx f;
+    uint32_t zero[2 * MAXL] = {0};
+    if (init_ctx(&f, L, 2, p, beta, zero)) return -1;
+    fe_mul(&f, r, x, y);
+    return 0;
+}
+
 int oracle_fp_mul(int L, const uint32_t *p, const uint32_t *x, const uint32_t *y, uint32_t *r) {
     fctx f;
     uint32_t zero[MAXL] = {0};
-    if (init_ctx(&f, L, p, zero)) return -1;
+    if (init_ctx(&f, L, 1, p, NULL, zero)) return -1;
     fp_mul(&f, r, x, y);
     return 0;
 }
@@ -421,7 +508,7 @@ int oracle_fp_mul(int L, const uint32_t *p, const uint32_t *x, const uint32_t *y
 int oracle_fp_inv(int L, const uint32_t *p, const uint32_t *x, uint32_t *r) {
     fctx f;
     uint32_t zero[MAXL] = {0};
-    if (init_ctx(&f, L, p, zero)) return -1;
+    if (init_ctx(&f, L, 1, p, NULL, zero)) return -1;
     if (bn_is_zero(x, L)) return -3;
     fp_inv(&f, r, x);
     return 0;

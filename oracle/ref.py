@@ -1,4 +1,4 @@
-"""Python-int oracle for the G1 MSM — TEST INFRASTRUCTURE ONLY.
+"""Python-int oracle for the G1 / G2 MSM — TEST INFRASTRUCTURE ONLY.
 
 Only tests/, __graft_entry__.smoke() and bench.py's cpu_baseline / --impl
 reference legs may import this module.  The product path never does.
@@ -34,23 +34,74 @@ def inv_mod(x: int, p: int) -> int:
     return pow(x, -1, p)
 
 
+class Fp:
+    """F_p on Python ints (G1)."""
+
+    def __init__(self, p: int):
+        self.p = p
+        self.zero, self.one = 0, 1
+
+    def add(self, x, y): return (x + y) % self.p
+    def sub(self, x, y): return (x - y) % self.p
+    def mul(self, x, y): return x * y % self.p
+    def neg(self, x): return (-x) % self.p
+    def inv(self, x): return inv_mod(x, self.p)
+    def small(self, k: int): return k % self.p
+    def elem(self, v): return v % self.p
+
+
+class Fp2:
+    """F_p^2 = F_p[u]/(u^2 - beta), elements (c0, c1) = c0 + c1 u (G2).  The
+    product is the schoolbook polynomial product reduced by u^2 = beta."""
+
+    def __init__(self, p: int, beta: int):
+        self.p, self.beta = p, beta
+        self.zero, self.one = (0, 0), (1, 0)
+
+    def add(self, x, y): return ((x[0] + y[0]) % self.p, (x[1] + y[1]) % self.p)
+    def sub(self, x, y): return ((x[0] - y[0]) % self.p, (x[1] - y[1]) % self.p)
+    def neg(self, x): return ((-x[0]) % self.p, (-x[1]) % self.p)
+
+    def mul(self, x, y):
+        p = self.p
+        return ((x[0] * y[0] + self.beta * x[1] * y[1]) % p, (x[0] * y[1] + x[1] * y[0]) % p)
+
+    def inv(self, x):
+        # (x0 + x1 u)^-1 = (x0 - x1 u) / (x0^2 - beta x1^2), the norm lies in F_p
+        p = self.p
+        nrm = (x[0] * x[0] - self.beta * x[1] * x[1]) % p
+        ni = inv_mod(nrm, p)
+        return (x[0] * ni % p, (-x[1]) * ni % p)
+
+    def small(self, k: int): return (k % self.p, 0)
+    def elem(self, v): return (v[0] % self.p, v[1] % self.p)
+
+
+def field(c) -> "Fp | Fp2":
+    c = get(c)
+    return Fp2(c.p, c.beta) if c.deg == 2 else Fp(c.p)
+
+
 def on_curve(c: Curve, P: Point) -> bool:
     if P is None:
         return True
+    F = field(c)
     x, y = P
-    return (y * y - (x * x * x + c.a * x + c.b)) % c.p == 0
+    rhs = F.add(F.add(F.mul(F.mul(x, x), x), F.mul(F.elem(c.a), x)), F.elem(c.b))
+    return F.mul(y, y) == rhs
 
 
 def neg(c: Curve, P: Point) -> Point:
     if P is None:
         return None
-    return (P[0], (-P[1]) % c.p)
+    return (P[0], field(c).neg(P[1]))
 
 
 def add(c: Curve, P: Point, Q: Point) -> Point:
     """Affine chord-and-tangent addition with every exceptional case explicit
-    ("PADD ... including point doubling", PAPER.md:116 footnote 2)."""
-    p = c.p
+    ("PADD ... including point doubling", PAPER.md:116 footnote 2), over F_p
+    (G1) or F_p^2 (G2)."""
+    F = field(c)
     if P is None:
         return Q
     if Q is None:
@@ -58,13 +109,14 @@ def add(c: Curve, P: Point, Q: Point) -> Point:
     x1, y1 = P
     x2, y2 = Q
     if x1 == x2:
-        if (y1 + y2) % p == 0:          # P == -Q (covers y == 0 doubling too)
+        if F.add(y1, y2) == F.zero:      # P == -Q (covers y == 0 doubling too)
             return None
-        lam = (3 * x1 * x1 + c.a) * inv_mod(2 * y1, p) % p   # tangent
+        num = F.add(F.mul(F.small(3), F.mul(x1, x1)), F.elem(c.a))   # tangent
+        lam = F.mul(num, F.inv(F.add(y1, y1)))
     else:
-        lam = (y2 - y1) * inv_mod(x2 - x1, p) % p             # chord
-    x3 = (lam * lam - x1 - x2) % p
-    y3 = (lam * (x1 - x3) - y1) % p
+        lam = F.mul(F.sub(y2, y1), F.inv(F.sub(x2, x1)))             # chord
+    x3 = F.sub(F.sub(F.mul(lam, lam), x1), x2)
+    y3 = F.sub(F.mul(lam, F.sub(x1, x3)), y1)
     return (x3, y3)
 
 
@@ -99,21 +151,25 @@ def generator(c) -> Point:
 # ---- wire encoding (the ABI's: little-endian u32 limbs, identity = (0,0)) ----
 
 def encode_point(c, P: Point) -> list:
+    """x || y; a G2 coordinate is c0 || c1 (each L limbs)."""
     c = get(c)
     L = c.limbs
     if P is None:
-        return [0] * (2 * L)
+        return [0] * (2 * c.coord_limbs)
+    if c.deg == 2:
+        return [w for v in (P[0][0], P[0][1], P[1][0], P[1][1]) for w in int_to_limbs(v, L)]
     return int_to_limbs(P[0], L) + int_to_limbs(P[1], L)
 
 
 def decode_point(c, limbs: Sequence[int]) -> Point:
     c = get(c)
     L = c.limbs
-    x = limbs_to_int(limbs[:L])
-    y = limbs_to_int(limbs[L:2 * L])
-    if x == 0 and y == 0:
+    v = [limbs_to_int(limbs[i * L:(i + 1) * L]) for i in range(2 * c.deg)]
+    if not any(v):
         return None
-    return (x, y)
+    if c.deg == 2:
+        return ((v[0], v[1]), (v[2], v[3]))
+    return (v[0], v[1])
 
 
 def int_to_limbs(v: int, n: int) -> list:

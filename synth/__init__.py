@@ -29,7 +29,10 @@ ORDERS = {
     "toy_a0": (14, 9967),
     "toy_a2": (14, 10091),
 }
-CURVE_IDS = {"bn254": 0, "bls12_381": 1, "mnt4_753": 2, "toy_a0": 100, "toy_a2": 101}
+ORDERS["bn254_g2"] = ORDERS["bn254"]            # G2 shares r with G1
+ORDERS["bls12_381_g2"] = ORDERS["bls12_381"]
+CURVE_IDS = {"bn254": 0, "bls12_381": 1, "mnt4_753": 2, "toy_a0": 100, "toy_a2": 101,
+             "bn254_g2": 3, "bls12_381_g2": 4}
 NAMES = {v: k for k, v in CURVE_IDS.items()}
 
 DISTS = ("uniform", "zcash_like", "full_bits", "all_zero", "all_one", "r_minus_1",
@@ -157,4 +160,5 @@ def scalar_seed(config: int) -> int:
 
 
 def dlog_seed(curve) -> int:
-    return 2000 + {"bn254": 0, "bls12_381": 1, "mnt4_753": 2, "toy_a0": 3, "toy_a2": 4}[_name(curve)]
+    return 2000 + {"bn254": 0, "bls12_381": 1, "mnt4_753": 2, "toy_a0": 3, "toy_a2": 4,
+                   "bn254_g2": 5, "bls12_381_g2": 6}[_name(curve)]
