@@ -59,6 +59,8 @@ def lib():
                                     ctypes.c_uint64, u32p, ctypes.c_int],
             "oracle_ec_add_ext": [ctypes.c_int, ctypes.c_int, u32p, u32p, u32p, u32p, u32p, u32p],
             "oracle_fp2_mul": [ctypes.c_int, u32p, u32p, u32p, u32p, u32p],
+            "oracle_poly_eval": [ctypes.c_int, u32p, u32p, ctypes.c_uint64, u32p, ctypes.c_int, u32p,
+                                 ctypes.c_int],
             "oracle_fp_mul": [ctypes.c_int, u32p, u32p, u32p, u32p],
             "oracle_fp_inv": [ctypes.c_int, u32p, u32p, u32p],
             "oracle_bn_mod": [u32p, ctypes.c_int, u32p, ctypes.c_int, u32p],
@@ -199,6 +201,22 @@ def bn_mod(u: int, m: int, v: int, n: int) -> int:
     return ref.limbs_to_int(out)
 
 
+def poly_eval(curve, coeffs: np.ndarray, xs, nthreads: int | None = None) -> list:
+    """A(x) mod r for every x in xs (C oracle, Horner; the NTT definition,
+    PAPER.md:128).  coeffs: [N, Ls] u32 canonical (< r) scalar-field values of
+    `curve`."""
+    c = get(curve)
+    Ls = c.scalar_limbs
+    coeffs = _u32(coeffs).reshape(-1, Ls)
+    r = _u32(ref.int_to_limbs(c.r, Ls))
+    X = _u32([ref.int_to_limbs(x % c.r, Ls) for x in xs]).reshape(-1, Ls)
+    out = np.zeros((X.shape[0], Ls), dtype=np.uint32)
+    if lib().oracle_poly_eval(Ls, _p(r), _p(coeffs), coeffs.shape[0], _p(X), X.shape[0], _p(out),
+                              nthreads or default_threads()):
+        raise RuntimeError("oracle_poly_eval failed")
+    return [ref.limbs_to_int(row) for row in out]
+
+
 def closed_form(curve, scalars: np.ndarray, dlogs: np.ndarray) -> np.ndarray:
     """sum_i k_i (a_i G) = (sum_i k_i a_i mod r) G  (SURVEY.md §8(c) pins).
 
@@ -232,4 +250,4 @@ def dot_mod(scalars: np.ndarray, dlogs: np.ndarray, r: int) -> int:
 
 
 __all__ = ["curves", "ref", "msm", "mul_each", "points_from_dlogs", "closed_form", "dot_mod",
-           "ec_add", "fp_mul", "fp2_mul", "fp_inv", "bn_mod", "build", "default_threads", "generator_limbs"]
+           "ec_add", "fp_mul", "fp2_mul", "fp_inv", "poly_eval", "bn_mod", "build", "default_threads", "generator_limbs"]

@@ -514,6 +514,62 @@ int oracle_fp_inv(int L, const uint32_t *p, const uint32_t *x, uint32_t *r) {
     return 0;
 }
 
+/* ------------------------------------------------ NTT definition (NEXT-4) */
+/* a_k = A(x_k) = sum_i A_i x_k^i over F_r by Horner's rule (PAPER.md:128
+ * §2.2: the N-NTT is the evaluation of A at the powers of w_N).  One output
+ * per call of horner(); threads split the evaluation points. */
+typedef struct {
+    const fctx *f;
+    const uint32_t *coeffs, *xs;
+    uint64_t n;
+    int begin, end;
+    uint32_t *out;
+} ejob;
+
+static void *run_eval(void *arg) {
+    ejob *j = (ejob *)arg;
+    const fctx *f = j->f;
+    int L = f->L;
+    for (int q = j->begin; q < j->end; ++q) {
+        uint32_t acc[MAXL];
+        memset(acc, 0, sizeof(acc));
+        for (uint64_t i = j->n; i-- > 0;) {
+            fp_mul(f, acc, acc, j->xs + (size_t)q * L);
+            fp_add(f, acc, acc, j->coeffs + (size_t)i * L);
+        }
+        memcpy(j->out + (size_t)q * L, acc, sizeof(uint32_t) * L);
+    }
+    return NULL;
+}
+
+/* out[q] = A(xs[q]) mod r, q < m; coeffs: n x L limbs (< r), xs: m x L limbs */
+int oracle_poly_eval(int L, const uint32_t *r, const uint32_t *coeffs, uint64_t n, const uint32_t *xs,
+                     int m, uint32_t *out, int nthreads) {
+    fctx f;
+    uint32_t zero[MAXL] = {0};
+    if (init_ctx(&f, L, 1, r, NULL, zero)) return -1;
+    if (nthreads < 1) nthreads = 1;
+    if (nthreads > m) nthreads = m > 0 ? m : 1;
+    ejob *jobs = (ejob *)calloc(nthreads, sizeof(ejob));
+    pthread_t *th = (pthread_t *)calloc(nthreads, sizeof(pthread_t));
+    if (!jobs || !th) { free(jobs); free(th); return -2; }
+    int chunk = (m + nthreads - 1) / nthreads;
+    for (int t = 0; t < nthreads; ++t) {
+        jobs[t].f = &f;
+        jobs[t].coeffs = coeffs;
+        jobs[t].xs = xs;
+        jobs[t].n = n;
+        jobs[t].begin = t * chunk < m ? t * chunk : m;
+        jobs[t].end = (t + 1) * chunk < m ? (t + 1) * chunk : m;
+        jobs[t].out = out;
+        pthread_create(&th[t], NULL, run_eval, &jobs[t]);
+    }
+    for (int t = 0; t < nthreads; ++t) pthread_join(th[t], NULL);
+    free(jobs);
+    free(th);
+    return 0;
+}
+
 /* r = u mod v (Knuth D), exported so the tests can pin it against Python ints */
 int oracle_bn_mod(const uint32_t *u, int m, const uint32_t *v, int n, uint32_t *r) {
     if (n < 1 || n > MAXL || m < n || m > 2 * MAXL || v[n - 1] == 0) return -1;
