@@ -37,9 +37,22 @@ def _newest(paths):
     return max(os.path.getmtime(p) for p in paths)
 
 
+def _deps(obj: str, src: str):
+    """Headers a TU includes, from the depfile nvcc wrote next to the object
+    (all headers when there is none yet)."""
+    dep = obj[:-2] + ".d"
+    try:
+        with open(dep) as f:
+            text = f.read().replace("\\\n", " ")
+        files = [w for w in text.split(":", 1)[1].split() if os.path.exists(w)]
+        return files + [src]
+    except (OSError, IndexError):
+        return _headers() + [src]
+
+
 def _compile(src: str, verbose: bool) -> str:
     obj = os.path.join(BUILD, os.path.basename(src)[:-3] + ".o")
-    cmd = [NVCC, *ARCH, *FLAGS, "-c", src, "-o", obj]
+    cmd = [NVCC, *ARCH, *FLAGS, "-MD", "-MF", obj[:-2] + ".d", "-c", src, "-o", obj]
     if verbose:
         cmd += ["-Xptxas", "-v"]
     r = subprocess.run(cmd, capture_output=True, text=True)
@@ -56,13 +69,12 @@ def build(force: bool = False, verbose: bool = False) -> str:
     if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= _newest(deps):
         return LIB
     os.makedirs(BUILD, exist_ok=True)
-    hdr_time = _newest(_headers())
     todo = []
     objs = []
     for s in srcs:
         obj = os.path.join(BUILD, os.path.basename(s)[:-3] + ".o")
         objs.append(obj)
-        if force or verbose or not os.path.exists(obj) or os.path.getmtime(obj) < max(hdr_time, os.path.getmtime(s)):
+        if force or verbose or not os.path.exists(obj) or os.path.getmtime(obj) < _newest(_deps(obj, s)):
             todo.append(s)
     with cf.ThreadPoolExecutor(max_workers=max(1, min(len(todo), os.cpu_count() or 4))) as ex:
         list(ex.map(lambda s: _compile(s, verbose), todo))

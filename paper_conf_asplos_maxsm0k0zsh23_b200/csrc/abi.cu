@@ -96,6 +96,8 @@ const CurveImpl* impl_for(int curve) {
     case GZKP_MNT4_753: return impl_mnt4_753();
     case GZKP_TOY_A0: return impl_toy_a0();
     case GZKP_TOY_A2: return impl_toy_a2();
+    case GZKP_BN254_G2: return impl_bn254_g2();
+    case GZKP_BLS12_381_G2: return impl_bls12_381_g2();
     default: return nullptr;
   }
 }
@@ -482,7 +484,7 @@ gzkp_status gzkp_field_op(int curve, int op, const void* a, const void* b, void*
   init_pool_once();
   const CurveImpl* c = impl_for(curve);
   if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
-  if (op < 0 || op > 5 || (n && (!a || !b || !out))) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
+  if (op < 0 || op > 6 || (n && (!a || !b || !out))) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
   return c->field_op(op, a, b, out, n, (cudaStream_t)stream);
 }
 

@@ -14,6 +14,7 @@
 // field value is canonical, so the P == Q tests are exact limb comparisons.
 #pragma once
 #include "field.cuh"
+#include "field2.cuh"
 #include "field_dfp.cuh"
 
 namespace gzkp {
@@ -21,7 +22,7 @@ namespace gzkp {
 template <class C>
 struct EC {
   static constexpr int N = C::N;
-  using Fp = F<C>;
+  using Fp = Field<C>;
 
   struct Xyzz {
     uint32_t X[N], Y[N], ZZ[N], ZZZ[N];
@@ -247,7 +248,7 @@ struct EC {
 template <class C>
 struct CoopEC {
   static constexpr int N = C::N;
-  using Fp = F<C>;
+  using Fp = Field<C>;
   using E = EC<C>;
   using Xyzz = typename E::Xyzz;
 

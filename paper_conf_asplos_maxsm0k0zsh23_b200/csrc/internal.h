@@ -59,6 +59,8 @@ const CurveImpl* impl_bls12_381();
 const CurveImpl* impl_mnt4_753();
 const CurveImpl* impl_toy_a0();
 const CurveImpl* impl_toy_a2();
+const CurveImpl* impl_bn254_g2();
+const CurveImpl* impl_bls12_381_g2();
 const CurveImpl* impl_for(int curve);
 
 gzkp_status set_error(gzkp_status st, const std::string& msg);

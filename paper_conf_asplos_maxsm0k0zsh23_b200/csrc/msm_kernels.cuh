@@ -49,7 +49,7 @@ GZ_DEV uint32_t digit_code(int d) { return d ? ((uint32_t)abs(d) | (d < 0 ? VAL_
 // ------------------------------------------------------------ a1 to_mont
 template <class C>
 __global__ void k_to_mont(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, size_t n) {
-  using Fp = F<C>;
+  using Fp = Field<C>;
   using E = EC<C>;
   constexpr int N = C::N;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
@@ -285,7 +285,7 @@ template <class C, bool MIXED = false>
 __global__ void __launch_bounds__(128, AccumCfg<C>::MIN_CTAS)
     k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off, Group grp,
             const uint32_t* __restrict__ pts, int S, uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay) {
-  using Fp = F<C>;
+  using Fp = Field<C>;
   using EC_ = EC<C>;
   using St = Stage<C>;
   constexpr int N = C::N;
@@ -573,7 +573,7 @@ __global__ void k_combine(const uint32_t* __restrict__ partials, int count, uint
 template <class C>
 __global__ void __launch_bounds__(128) k_precompute_step(const uint32_t* __restrict__ prev, uint32_t* __restrict__ next,
                                                          size_t n, int c) {
-  using Fp = F<C>;
+  using Fp = Field<C>;
   using EC_ = EC<C>;
   constexpr int N = C::N;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
@@ -603,7 +603,7 @@ __global__ void __launch_bounds__(128) k_precompute_step(const uint32_t* __restr
 template <class C>
 __global__ void __launch_bounds__(128) k_fixed_base(const uint32_t* __restrict__ sc, size_t n,
                                                     uint32_t* __restrict__ out) {
-  using Fp = F<C>;
+  using Fp = Field<C>;
   using EC_ = EC<C>;
   constexpr int N = C::N;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
@@ -636,7 +636,7 @@ __global__ void __launch_bounds__(128) k_fixed_base(const uint32_t* __restrict__
 template <class C>
 __global__ void k_field_op(int op, const uint32_t* __restrict__ a, const uint32_t* __restrict__ b,
                            uint32_t* __restrict__ out, size_t n) {
-  using Fp = F<C>;
+  using Fp = Field<C>;
   using EC_ = EC<C>;
   constexpr int N = C::N;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
@@ -663,7 +663,7 @@ __global__ void k_field_op(int op, const uint32_t* __restrict__ a, const uint32_
 template <class C>
 __global__ void k_ec_op(int op, const uint32_t* __restrict__ P, const uint32_t* __restrict__ Q,
                         uint32_t* __restrict__ out, size_t n) {
-  using Fp = F<C>;
+  using Fp = Field<C>;
   using EC_ = EC<C>;
   constexpr int N = C::N;
   for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {

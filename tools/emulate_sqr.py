@@ -90,7 +90,11 @@ def limbs(v, N):
 for name, p in [("bn254", 0x30644e72e131a029b85045b68181585d97816a916871ca8d3c208c16d87cfd47),
                 ("bls", 0x1a0111ea397fe69a4b1ba7b6434bacd764774b84f38512bf6730d2a0f6b0f6241eabfffeb153ffffb9feffffffffaaab),
                 ("mnt4", 0x1c4c62d92c41110229022eee2cdadb7f997505b8fafed5eb7e8f96c97d87307fdb925e8a0ed8d99d124d9a15af79db117e776f218059db80f0da5cb537e38685acce9767254a4638810719ac425f0e39d54522cdd119f5e9063de245e8001),
-                ("toy", 10099)]:
+                ("toy", 10099),
+                # scalar fields F_r (NTT, NEXT-4): BLS12-381's r has a single spare bit
+                ("r_bn254", 0x30644e72e131a029b85045b68181585d2833e84879b9709143e1f593f0000001),
+                ("r_bls", 0x73eda753299d7d483339d80809a1d80553bda402fffe5bfeffffffff00000001),
+                ("r_mnt4", 0x1c4c62d92c41110229022eee2cdadb7f997505b8fafed5eb7e8f96c97d87307fdb925e8a0ed8d99d124d9a15af79db26c5c28c859a99b3eebca9429212636b9dff97634993aa4d6c381bc3f0057974ea099170fa13a4fd90776e240000001)]:
     N = (p.bit_length() + 31) // 32
     N += N & 1
     n0 = (-pow(p, -1, 1 << 32)) % (1 << 32)
