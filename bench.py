@@ -45,15 +45,33 @@ WORKLOADS = {
     "bls12_381_2p26_sparse": ("bls12_381", 26, 5, "zcash_like", "BLS12-381 G1 MSM n=2^26, sparse/skewed scalars"),
     "bls12_381_2p26": ("bls12_381", 26, 6, "uniform", "BLS12-381 G1 MSM n=2^26, uniform scalars"),
     "bn254_2p10": ("bn254", 10, 1, "uniform", "BN254 G1 MSM n=2^10, uniform random scalars"),
+    # G2 (not a BASELINE config: the same MSM over F_p^2)
+    "bn254_g2_2p20": ("bn254_g2", 20, 7, "uniform", "BN254 G2 MSM n=2^20, uniform scalars (NEXT-3)"),
+    "bls12_381_g2_2p20": ("bls12_381_g2", 20, 8, "uniform", "BLS12-381 G2 MSM n=2^20, uniform scalars (NEXT-3)"),
 }
-L_BY_CURVE = {"bn254": 8, "bls12_381": 12, "mnt4_753": 24}
-METRIC = "G1 MSM points/sec"
+# NTT workloads (Table 5 sizes): field, log2 N, seed config
+NTT_WORKLOADS = {
+    "bls12_381_ntt_2p24": ("bls12_381", 24, 9, "BLS12-381 F_r (256-bit) 2^24-NTT (PAPER.md Table 5)"),
+    "bn254_ntt_2p22": ("bn254", 22, 10, "BN254 F_r 2^22-NTT"),
+    "mnt4_753_ntt_2p20": ("mnt4_753", 20, 11, "MNT4-753 F_r (753-bit) 2^20-NTT (PAPER.md Table 5)"),
+}
+# u32 words of one curve coordinate (G2: two F_p limbs sets c0 || c1)
+L_BY_CURVE = {"bn254": 8, "bls12_381": 12, "mnt4_753": 24, "bn254_g2": 16, "bls12_381_g2": 24}
 L2_BYTES = 126 * 1024 * 1024
 
 
-def madd_imad(L: int) -> int:
+def metric_for(curve: str) -> str:
+    return ("G2" if curve.endswith("_g2") else "G1") + " MSM points/sec"
+
+
+def madd_imad(L: int, g2: bool = False) -> int:
     """Algorithmic IMAD count of one XYZZ mixed add:
-    madd = 8M + 2S with M = 4L^2 + L, S = 3L^2 + 2L."""
+    madd = 8M + 2S with M = 4L^2 + L, S = 3L^2 + 2L over F_p (L limbs).
+    G2 (L = 2 x base limbs): an F_p^2 product is 3 base products (Karatsuba)
+    and a square 2, so madd = 8 (3M) + 2 (2M) = 28M."""
+    if g2:
+        Lb = L // 2
+        return 28 * (4 * Lb * Lb + Lb)
     return 8 * (4 * L * L + L) + 2 * (3 * L * L + 2 * L)
 
 
@@ -173,7 +191,7 @@ def run_reference(args, wl):
         walls.append(wall)
     value = n_s * len(walls) / sum(walls)
     line = {
-        "impl": "reference", "metric": METRIC, "value": value, "unit": "points/s", "n_gpus": args.gpus,
+        "impl": "reference", "metric": metric_for(curve), "value": value, "unit": "points/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(walls) / len(walls),
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32 (exact F_p)",
         "data": "synthetic",
@@ -187,6 +205,168 @@ def run_reference(args, wl):
     print(json.dumps(line), flush=True)
 
 
+# ------------------------------------------------------------ NTT (NEXT-4)
+
+def ntt_oracle_rate(field: str, k: np.ndarray, log_n: int, budget_s: float):
+    """The oracle's NTT throughput: outputs a_k = A(w^k) computed one by one by
+    Horner over all N coefficients (the definition, O(N) per output), on all
+    host cores.  Linear in the number of outputs, so m outputs in t seconds is
+    a rate of m / t elements/s for the full-size transform."""
+    import oracle
+    from oracle import curves as oc, ntt as ontt
+    c = oc.get(field)
+    cores = oracle.default_threads()
+    w = ontt.root_of_unity(c, log_n)
+    t0 = time.perf_counter()
+    oracle.poly_eval(c, k, [w], nthreads=1)
+    one = max(time.perf_counter() - t0, 1e-6)
+    m = max(cores, int(budget_s / one) * cores)
+    m = min(m, 4096)
+    xs = [pow(w, j, c.r) for j in range(m)]
+    t0 = time.perf_counter()
+    oracle.poly_eval(c, k, xs, nthreads=cores)
+    wall = time.perf_counter() - t0
+    return m / wall, wall, cores, m
+
+
+def run_ntt_reference(args, wl):
+    world, rank, _ = dist_env()
+    field, logn, cfg, desc = NTT_WORKLOADS[wl]
+    if rank != 0:
+        return
+    k = synth.scalars(field, 1 << logn, synth.scalar_seed(cfg))
+    per_step = max(2.0, 60.0 / (args.steps + args.warmup))
+    for _ in range(args.warmup):
+        ntt_oracle_rate(field, k, logn, per_step / 4)
+    rates, walls = [], []
+    for _ in range(args.steps):
+        rate, wall, cores, m = ntt_oracle_rate(field, k, logn, per_step)
+        rates.append(rate)
+        walls.append(wall)
+    value = statistics.median(rates)
+    line = {"impl": "reference", "metric": "F_r NTT elements/sec", "value": value, "unit": "elements/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": 1e3 * (1 << logn) / value, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "u32 (exact F_r)", "data": "synthetic",
+            "config": {"workload": wl, "field": field, "log_n": logn, "baseline_config": desc},
+            "cpu_baseline": {"value": value, "unit": "elements/s", "cores": cores, "kind": "oracle",
+                             "sample": f"{m} outputs A(w^k) of the 2^{logn} transform per step, Horner over "
+                                       f"all coefficients (oracle.c), {statistics.median(walls):.1f} s"},
+            "e2e": {"value": value, "unit": "elements/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_ntt(args, wl):
+    """One step = one forward 2^logn-NTT over F_r, inputs resident in HBM.  N > 1
+    GPUs: independent transforms per rank (replicas: one NTT does not shard
+    without an all-to-all the paper does not use), value = total elements/s."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_asplos_maxsm0k0zsh23_b200 as gz
+    from paper_conf_asplos_maxsm0k0zsh23_b200 import build as gbuild
+
+    world, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if not os.path.exists(gz.LIB_PATH) and rank == 0:
+        gbuild.build()
+    if world > 1:
+        dist.barrier()
+    field, logn, cfg, desc = NTT_WORKLOADS[wl]
+    n = 1 << logn
+    ks = synth.scalars(field, n, synth.scalar_seed(cfg) + rank)
+    Ls = ks.shape[1]
+    A = gz.to_device(ks)
+    out = torch.empty_like(A)
+    stream = torch.cuda.current_stream()
+    nbytes = n * Ls * 4
+    flush = nbytes < 2 * L2_BYTES
+    flush_buf = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device="cuda") if flush else None
+    for _ in range(args.warmup):
+        gz.ntt(field, A, out=out)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    sampler = ClockSampler(local)
+    sampler.start()
+    time.sleep(0.3)
+    torch.cuda.synchronize()
+    total_ms = 0.0
+    for _ in range(args.steps):
+        if flush:
+            flush_buf.zero_()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        gz.ntt(field, A, out=out)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        total_ms += e0.elapsed_time(e1)
+    clocks = sampler.stop()
+    t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms = float(t.item()) / args.steps
+    value = world * n / (ms / 1e3)
+    launches = gz.ntt_last_launches()
+    # roofline: the passes (k_ntt_pass) ARE the step; algorithmic work =
+    # (N/2) log N butterflies x one F_r Montgomery product (4L^2 + L IMAD)
+    peaks, src = load_peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    M = 4 * Ls * Ls + Ls
+    imad = (n // 2) * logn * M
+    peak = 148 * 64 * sm_max * 1e6
+    achieved = imad / (ms / 1e3)
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "ntt_traffic.json")) as f:
+            traffic = json.load(f).get(wl)
+    except Exception:
+        pass
+    roofline = {"bound": "alu", "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "TIMAD/s",
+                "frac": achieved / peak, "traffic": traffic, "kernel": f"k_ntt_pass x {launches} passes",
+                "algorithmic": f"(N/2) log N = {(n // 2) * logn} butterflies x {M} IMAD (one F_r product)",
+                "peak_src": f"148 SM x 64 IMAD/clk x {sm_max:.0f} MHz ({src} sm_max)",
+                "hbm_bytes_algorithmic": 2 * nbytes}
+    e2e = None
+    if not args.no_e2e:
+        Ah = A.cpu().pin_memory()
+        Oh = torch.empty_like(Ah).pin_memory()
+        Ad = torch.empty_like(A)
+        k_e2e = max(1, min(args.steps, 5))
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        for _ in range(k_e2e):
+            Ad.copy_(Ah, non_blocking=True)
+            gz.ntt(field, Ad, out=Ad)
+            Oh.copy_(Ad, non_blocking=True)
+            torch.cuda.synchronize()
+        e2e_ms = (time.perf_counter() - t0) * 1e3 / k_e2e
+        e2e = {"value": world * n / (e2e_ms / 1e3), "unit": "elements/s", "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": nbytes * world, "d2h_bytes_per_step": nbytes * world,
+               "api": "H2D + gzkp_ntt (in place) + D2H"}
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        rate, wall, cores, m = ntt_oracle_rate(field, ks, logn, 10.0)
+        cpu = {"value": rate, "unit": "elements/s", "cores": cores, "kind": "oracle",
+               "sample": f"{m} outputs of the 2^{logn} transform, each A(w^k) by Horner over all "
+                         f"coefficients (oracle.c), wall {wall:.1f} s"}
+    if rank == 0:
+        line = {"metric": "F_r NTT elements/sec", "value": value, "unit": "elements/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "u32 (exact F_r, Montgomery)",
+                "data": "synthetic (seeded coefficients uniform in [0, r))",
+                "config": {"workload": wl, "field": field, "log_n": logn, "baseline_config": desc,
+                           "parallelism": f"replicas{world}" if world > 1 else "single",
+                           "l2": "flushed between steps" if flush else f"input {nbytes >> 20} MiB > L2"},
+                "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks,
+                "gpu_launches": launches * args.steps}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
 # ---------------------------------------------------------------- GPU arm
 
 def main():
@@ -195,7 +375,7 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="gzkp", choices=["gzkp", "reference"])
-    ap.add_argument("--workload", default="bls12_381_2p22", choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default="bls12_381_2p22", choices=sorted(WORKLOADS) + sorted(NTT_WORKLOADS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-prepared", action="store_true")
@@ -206,6 +386,12 @@ def main():
     args.warmup = max(args.warmup, 3)
     wl = args.workload
 
+    if wl in NTT_WORKLOADS:
+        if args.impl == "reference":
+            run_ntt_reference(args, wl)
+        else:
+            run_ntt(args, wl)
+        return
     if args.impl == "reference":
         run_reference(args, wl)
         return
@@ -231,6 +417,7 @@ def main():
     curve, logn, cfg, sdist, desc = WORKLOADS[wl]
     n = 1 << logn
     L = L_BY_CURVE[curve]
+    g2 = curve.endswith("_g2")
     lo, hi = gz.shard_range(n, world, rank)
     n_loc = hi - lo
 
@@ -332,7 +519,7 @@ def main():
         p_ms = pe0.elapsed_time(pe1) / args.steps
         pcalls = max(1, pprof["calls"])
         p_accum = pprof["phase_ms"]["accumulate"] / pcalls
-        p_ach = pprof["entries"] * madd_imad(L) / (p_accum / 1e3) if p_accum > 0 else 0.0
+        p_ach = pprof["entries"] * madd_imad(L, g2) / (p_accum / 1e3) if p_accum > 0 else 0.0
         prepared = {"value": n / (p_ms / 1e3), "unit": "points/s", "ms_per_step": p_ms,
                     "window_bits": info["window_bits"], "windows": info["windows"],
                     "table_bytes": info["bytes"], "prepare_s": prep_s,
@@ -350,7 +537,7 @@ def main():
     calls = max(1, prof["calls"])
     accum_ms = prof["phase_ms"]["accumulate"] / calls
     entries = prof["entries"]
-    imad_per_launch = entries * madd_imad(L)
+    imad_per_launch = entries * madd_imad(L, g2)
     achieved = imad_per_launch / (accum_ms / 1e3) if accum_ms > 0 else 0.0
     peak = 148 * 64 * sm_max * 1e6
     traffic = None
@@ -363,7 +550,8 @@ def main():
     roofline = {"bound": "alu", "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "TIMAD/s",
                 "frac": achieved / peak if peak else None, "traffic": traffic,
                 "kernel": "k_accum (bucket accumulation, XYZZ madd)",
-                "algorithmic": f"{entries} bucket entries x {madd_imad(L)} IMAD (8M+2S, App. B)",
+                "algorithmic": f"{entries} bucket entries x {madd_imad(L, g2)} IMAD "
+                               + ("(8M+2S over F_p^2 = 28 F_p products)" if g2 else "(8M+2S, App. B)"),
                 "peak_src": f"148 SM x 64 IMAD/clk x {sm_max:.0f} MHz ({peaks_src} sm_max)",
                 "accum_ms": accum_ms, "phase_ms_per_step": phase_share}
     launches = int(prof["launches"]) + (1 if world > 1 else 0)
@@ -420,7 +608,7 @@ def main():
 
     if rank == 0:
         line = {
-            "metric": METRIC, "value": value, "unit": "points/s", "n_gpus": world, "steps": args.steps,
+            "metric": metric_for(curve), "value": value, "unit": "points/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u32 (exact F_p, Montgomery)",
             "data": "synthetic (seeded scalars; points a_i*G generated on device)",

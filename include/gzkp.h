@@ -59,6 +59,13 @@ typedef enum {
   GZKP_BN254 = 0,
   GZKP_BLS12_381 = 1,
   GZKP_MNT4_753 = 2,
+  /* G2: the order-r subgroup of the
+   * sextic twist E'(F_p^2): y^2 = x^3 + b' over F_p^2 = F_p[u]/(u^2 + 1),
+   * b' = 3/(9+u) (BN254, EIP-197) and 4(1+u) (BLS12-381).  A coordinate is
+   * c0 || c1 (c0 + c1 u), each an F_p value as above, so field_bytes = 64 | 96;
+   * scalars are the same F_r scalars as G1. */
+  GZKP_BN254_G2 = 3,
+  GZKP_BLS12_381_G2 = 4,
   GZKP_TOY_A0 = 100, /* y^2 = x^3 + 3 over F_10099, prime order 9967 (tests) */
   GZKP_TOY_A2 = 101  /* y^2 = x^3 + 2x + 30 over F_10007, prime order 10091 (tests) */
 } gzkp_curve;
@@ -75,7 +82,7 @@ typedef enum {
 typedef void *gzkp_stream; /* a cudaStream_t; NULL = legacy default stream */
 
 /* --- sizes ------------------------------------------------------------ */
-size_t gzkp_field_bytes(int curve);   /* one coordinate: 32 | 48 | 96 (8 for toys) */
+size_t gzkp_field_bytes(int curve);   /* one coordinate: 32 | 48 | 96 (8 for toys; G2: 64 | 96) */
 size_t gzkp_scalar_bytes(int curve);  /* one scalar:     32 | 32 | 96 (4 for toys) */
 size_t gzkp_partial_bytes(int curve); /* one XYZZ partial: 4 * field_bytes */
 
@@ -142,6 +149,26 @@ gzkp_status gzkp_comm_destroy(void *comm);
 gzkp_status gzkp_msm_sharded(int curve, const void *points_affine, const void *scalars,
                              size_t n_local, void *out, gzkp_stream stream, void *comm);
 
+/* --- NTT over the scalar field F_r -------------------
+ * The POLY stage of the prover (§2.2, §3): for N = 2^log_n and
+ * A_i in F_r of `curve` (G1 and G2 ids share F_r),
+ *   inverse = 0:  out[k] = sum_i in[i] w_N^(i k)        = A(w_N^k)
+ *   inverse = 1:  out[i] = N^-1 sum_k in[k] w_N^(-i k)
+ * with w_N = g^((r-1)/N), g the smallest quadratic non-residue mod r
+ * (reading R15; w_N^(N/2) = -1).  in/out: device, N elements of
+ * gzkp_scalar_bytes(curve) bytes each, canonical (< r) little-endian, 16-B
+ * aligned; in == out is allowed.  log_n <= gzkp_ntt_max_log(curve)
+ * (min(2-adicity of r - 1, 30): 28 | 30 | 30).  Enqueued on `stream`; twiddle
+ * tables are built on the device at the first call per (log_n, direction) and
+ * kept by the library.  Inputs >= r are not detected. */
+int gzkp_ntt_max_log(int curve);
+gzkp_status gzkp_ntt(int curve, const void *in, void *out, int log_n, int inverse, gzkp_stream stream);
+/* kernels launched by this thread's last gzkp_ntt call (benchmark bookkeeping) */
+int gzkp_ntt_last_launches(void);
+/* F_r element ops for the tests, same op codes as gzkp_field_op (0..5). */
+gzkp_status gzkp_scalar_field_op(int curve, int op, const void *a, const void *b, void *out, size_t n,
+                                 gzkp_stream stream);
+
 /* --- benchmark/test input generation (not on the MSM path) --------------- */
 /* out[i] = scalars[i] * G (canonical affine) for the curve's fixed generator G.
  * Used to build synthetic proving-key points with known discrete logs. */
@@ -151,7 +178,9 @@ gzkp_status gzkp_fixed_base_mul(int curve, const void *scalars, size_t n, void *
 /* --- diagnostics ----------------------------------------------------------- */
 /* Elementwise field ops on canonical inputs (device arrays of n elements):
  * op 0: a*b mod p, 1: a+b, 2: a-b, 3: a^-1 (a != 0), 4: round trip to/from Montgomery,
- * 5: a^2 mod p (the dedicated Montgomery squaring). */
+ * 5: a^2 mod p (the dedicated Montgomery squaring), 6: a*b mod p by the FP64
+ * (DFP) Montgomery product where the curve has one (BLS12-381, MNT4-753; NEXT-2),
+ * else the IMAD product.  For G2 curves the elements are F_p^2 values c0 || c1. */
 gzkp_status gzkp_field_op(int curve, int op, const void *a, const void *b, void *out, size_t n,
                           gzkp_stream stream);
 /* Elementwise group ops on canonical affine points (device, n points each):

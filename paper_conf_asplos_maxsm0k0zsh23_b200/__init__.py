@@ -17,7 +17,8 @@ import numpy as np
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libgzkp.so")
 
-CURVES = {"bn254": 0, "bls12_381": 1, "mnt4_753": 2, "toy_a0": 100, "toy_a2": 101}
+CURVES = {"bn254": 0, "bls12_381": 1, "mnt4_753": 2, "toy_a0": 100, "toy_a2": 101,
+          "bn254_g2": 3, "bls12_381_g2": 4}
 NAMES = {v: k for k, v in CURVES.items()}
 
 _lib = None
@@ -72,6 +73,10 @@ def lib():
             "gzkp_window_bits": ([i32, sz], i32),
             "gzkp_set_profiling": ([i32], i32),
             "gzkp_profile_read": ([ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_uint64), i32], i32),
+            "gzkp_ntt_max_log": ([i32], i32),
+            "gzkp_ntt": ([i32, vp, vp, i32, i32, vp], i32),
+            "gzkp_ntt_last_launches": ([], i32),
+            "gzkp_scalar_field_op": ([i32, i32, vp, vp, vp, sz, vp], i32),
             "gzkp_status_string": ([i32], ctypes.c_char_p),
             "gzkp_last_error": ([], ctypes.c_char_p),
         }
@@ -323,6 +328,48 @@ def ec_op(curve, op: int, P, Q, stream=None):
     return out
 
 
+# ------------------------------------------------------ NTT over F_r (NEXT-4)
+
+def ntt_max_log(curve) -> int:
+    return lib().gzkp_ntt_max_log(curve_id(curve))
+
+
+def ntt(curve, values, inverse: bool = False, out=None, stream=None):
+    """N-NTT over the scalar field of `curve`: out[k] = A(w_N^k),
+    or the inverse transform.  values: [N, Ls] u32 limbs (canonical < r) on
+    the device, N a power of two.  out may alias values."""
+    torch = _torch()
+    cid = curve_id(curve)
+    Ls = scalar_limbs(cid)
+    A = _dev_u32(values, Ls, "values")
+    n = A.shape[0]
+    log_n = n.bit_length() - 1
+    if n != 1 << log_n:
+        raise GzkpError("NTT size must be a power of two")
+    if out is None:
+        out = torch.empty_like(A)
+    _check(lib().gzkp_ntt(cid, A.data_ptr(), out.data_ptr(), log_n, 1 if inverse else 0, _stream_ptr(stream)),
+           "gzkp_ntt")
+    return out
+
+
+def ntt_last_launches() -> int:
+    return lib().gzkp_ntt_last_launches()
+
+
+def scalar_field_op(curve, op: int, a, b, stream=None):
+    """Elementwise F_r ops (same op codes as field_op) -- tests only."""
+    torch = _torch()
+    cid = curve_id(curve)
+    Ls = scalar_limbs(cid)
+    A = _dev_u32(a, Ls, "a")
+    B = _dev_u32(b, Ls, "b")
+    out = torch.empty_like(A)
+    _check(lib().gzkp_scalar_field_op(cid, op, A.data_ptr(), B.data_ptr(), out.data_ptr(), A.shape[0],
+                                      _stream_ptr(stream)), "gzkp_scalar_field_op")
+    return out
+
+
 # ------------------------------------------------------------- multi-GPU
 
 def broadcast_unique_id(rank: int, group=None) -> bytes:
@@ -380,4 +427,5 @@ def msm_sharded(curve, points_local, scalars_local, comm: Comm, out=None, stream
 
 __all__ = ["CURVES", "GzkpError", "lib", "msm", "msm_host", "PreparedPoints", "msm_partial", "combine_partials",
            "fixed_base_mul", "field_op", "ec_op", "Comm", "msm_sharded", "shard_range", "set_config",
-           "window_bits", "workspace_bytes", "set_profiling", "profile_read", "field_limbs", "scalar_limbs", "to_device", "to_numpy"]
+           "window_bits", "workspace_bytes", "set_profiling", "profile_read", "field_limbs", "scalar_limbs", "to_device",
+           "to_numpy", "ntt", "ntt_max_log", "ntt_last_launches", "scalar_field_op"]

@@ -103,7 +103,7 @@ const CurveImpl* impl_for(int curve) {
 }
 
 // the stream-ordered pool keeps freed workspace (no re-allocation per call)
-static void init_pool_once() {
+void init_pool_once() {
   static std::once_flag once;
   std::call_once(once, [] {
     int dev = 0;

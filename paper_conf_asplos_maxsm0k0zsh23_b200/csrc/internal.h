@@ -94,5 +94,8 @@ struct StreamCtx {
   int nev = 0;
 };
 gzkp_status stream_ctx(cudaStream_t s, StreamCtx** ctx);
+// once per process: stream-ordered pool release threshold, and a 4 KB
+// per-thread stack for the out-of-line MNT4-753 products (every entry point)
+void init_pool_once();
 
 }  // namespace gzkp
