@@ -30,17 +30,18 @@ struct Plan {
   uint32_t M = 0;        // Wb * B bucket keys
   int S = 64;            // entries per accumulation chunk
   int seg = 16;          // buckets per reduction segment
-  int heavy_levels = 0;  // depth of the heavy-bucket tree
+  int heavy_levels = 0;  // depth of the heavy-bucket tree (max over groups)
   size_t n = 0;
   uint64_t E_max = 0, chunks_max = 0;
   // workspace byte offsets
   size_t o_pts = 0, o_codes = 0, o_counts = 0, o_offsets = 0, o_cursor = 0, o_tiles = 0, o_vals = 0,
-         o_spay = 0, o_heavy = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_win = 0, total = 0;
+         o_spay = 0, o_heavy = 0, o_hlist = 0, o_hjobs = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_win = 0, total = 0;
   struct Grp {
     int t_lo, t_hi;             // windows (inclusive)
     uint32_t key_lo, key_hi;    // bucket keys
     uint64_t chunk_base, chunks_max;
     int heavy_levels;
+    uint32_t hmax, hbase;       // heavy-list capacity and first entry
     int seg = 16;               // reduction segment (buckets per thread)
   };
   std::vector<Grp> groups;
@@ -128,26 +129,27 @@ struct Impl {
     // g while group g+1 accumulates, so only the last group's post-processing
     // is exposed.  Weighted points share one bucket set: a single group.
     p.groups.clear();
+    // (Grp: t_lo, t_hi, key_lo, key_hi, chunk_base, chunks_max, heavy_levels, hmax, hbase)
     static const int pipeline = [] {
       const char* e = getenv("GZKP_PIPELINE");
       return e ? atoi(e) : 0;
     }();
     if (consolidated || !pipeline) {
-      p.groups.push_back({0, p.W - 1, 0, p.M, 0, 0, 0});
+      p.groups.push_back({0, p.W - 1, 0, p.M, 0, 0, 0, 0, 0});
     } else if (consolidated) {
-      p.groups.push_back({0, p.W - 1, 0, p.B, 0, 0, 0});
+      p.groups.push_back({0, p.W - 1, 0, p.B, 0, 0, 0, 0, 0});
     } else {
       int hi = p.W - 1;
       while (hi >= 0) {
         const int rem = hi + 1;
         const int sz = rem > 1 ? (rem + 1) / 2 : 1;
-        p.groups.push_back({hi - sz + 1, hi, (uint32_t)(hi - sz + 1) * p.B, (uint32_t)(hi + 1) * p.B, 0, 0, 0});
+        p.groups.push_back({hi - sz + 1, hi, (uint32_t)(hi - sz + 1) * p.B, (uint32_t)(hi + 1) * p.B, 0, 0, 0, 0, 0});
         hi -= sz;
       }
     }
     p.chunks_max = 0;
     p.heavy_levels = 0;
-    uint64_t seg_elems = 1, mid_elems = 1;
+    uint64_t seg_elems = 1, mid_elems = 1, hlist_elems = 0;
     for (auto& g : p.groups) {
       const uint64_t wins = consolidated ? (uint64_t)p.W : (uint64_t)(g.t_hi - g.t_lo + 1);
       const uint64_t bwins = consolidated ? 1 : wins;
@@ -165,8 +167,13 @@ struct Impl {
       mid_elems = std::max<uint64_t>(mid_elems, bwins * ((gsegs + WIN_PER_BLOCK - 1) / WIN_PER_BLOCK));
       g.chunk_base = p.chunks_max;
       g.chunks_max = (n * wins + p.S - 1) / p.S + 1;
+      // a heavy bucket spans > MERGE_QMAX chunks: at most chunks / MERGE_QMAX of them
+      g.hmax = (uint32_t)(g.chunks_max / MERGE_QMAX + 2);
+      g.hbase = (uint32_t)hlist_elems;
+      hlist_elems += g.hmax;
       g.heavy_levels = 0;
-      for (uint64_t span = 1; span < g.chunks_max; span *= HEAVY_FAN) ++g.heavy_levels;
+      for (uint64_t span = 1; span < g.chunks_max; span *= HEAVY_SPAN) ++g.heavy_levels;
+      p.heavy_levels = std::max(p.heavy_levels, g.heavy_levels);
       p.chunks_max += g.chunks_max;
     }
     const uint32_t G = p.B / p.seg;
@@ -181,6 +188,8 @@ struct Impl {
     p.o_vals = take(std::max<uint64_t>(p.E_max, 1) * 4);
     p.o_spay = take(2 * p.chunks_max * 4 * N * 4);
     p.o_heavy = take(4 * (p.groups.size() + 4));
+    p.o_hlist = take(16 * std::max<uint64_t>(hlist_elems, 1));
+    p.o_hjobs = take(4 * (size_t)std::max(p.heavy_levels, 1) * (hlist_elems + p.groups.size()));
     p.o_state = take(4 * N * 4);
     p.o_buckets = take((size_t)p.M * 4 * N * 4);
     (void)G;
@@ -304,6 +313,8 @@ struct Impl {
                                       (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
       GZ_CHECK(cudaFuncSetAttribute(k_reduce_win<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)((size_t)threads * 4 * N * 4)));
+      GZ_CHECK(cudaFuncSetAttribute(k_heavy_tree<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)((size_t)HEAVY_THREADS * 4 * N * 4)));
       attr_set = true;
     }
     // overlapped host->device path: the points are still arriving on another
@@ -340,15 +351,24 @@ struct Impl {
       uint32_t* heavy = U(p.o_heavy) + gi;
       const uint32_t nkeys = gr.key_hi - gr.key_lo;
       const int gm = (int)std::min<uint64_t>((nkeys + threads - 1) / threads, (uint64_t)sms * 16);
-      k_merge_bucket<C><<<gm, threads, 0, ss>>>(U(p.o_offsets), grp, p.S, U(p.o_spay), U(p.o_buckets), heavy);
+      uint4* hlist = (uint4*)U(p.o_hlist) + gr.hbase;
+      uint32_t* hjobs = U(p.o_hjobs) + (size_t)std::max(p.heavy_levels, 1) * (gr.hbase + gi);
+      k_merge_bucket<C><<<gm, threads, 0, ss>>>(U(p.o_offsets), grp, p.S, U(p.o_spay), U(p.o_buckets), heavy, hlist,
+                                                gr.hmax);
       GZ_CHECK(cudaGetLastError());
-      const int gh = (int)std::min<uint64_t>((gr.chunks_max + threads - 1) / threads, (uint64_t)sms * 8);
-      uint32_t stride = 1;
-      for (int l = 0; l < gr.heavy_levels; ++l, stride *= HEAVY_FAN) {
-        k_heavy_level<C><<<gh, threads, 0, ss>>>(U(p.o_offsets), grp, p.S, stride, heavy, U(p.o_spay));
+      if (gr.heavy_levels > 0) {
+        k_heavy_plan<<<1, 32, 0, ss>>>(heavy, hlist, gr.hmax, gr.heavy_levels, hjobs);
+        GZ_CHECK(cudaGetLastError());
+        ++launches;
+      }
+      const size_t hsmem = (size_t)HEAVY_THREADS * 4 * N * 4;
+      uint64_t stride = 1;
+      for (int l = 0; l < gr.heavy_levels; ++l, stride *= HEAVY_SPAN) {
+        k_heavy_tree<C><<<sms * 2, HEAVY_THREADS, hsmem, ss>>>(heavy, hlist, gr.hmax, hjobs + (size_t)l * (gr.hmax + 1),
+                                                             stride, grp, U(p.o_spay));
         GZ_CHECK(cudaGetLastError());
       }
-      k_heavy_final<C><<<gm, threads, 0, ss>>>(U(p.o_offsets), grp, p.S, heavy, U(p.o_spay), U(p.o_buckets));
+      k_heavy_final<C><<<sms, threads, 0, ss>>>(heavy, hlist, gr.hmax, grp, U(p.o_spay), U(p.o_buckets));
       GZ_CHECK(cudaGetLastError());
       launches += 2 + gr.heavy_levels;
       ev_merged = profile_event(prof, ss);

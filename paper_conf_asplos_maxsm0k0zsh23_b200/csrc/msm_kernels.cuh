@@ -21,7 +21,6 @@ namespace gzkp {
 
 constexpr uint32_t VAL_NEG = 0x80000000u;    // entry / digit-code flag: negative digit
 constexpr int MERGE_QMAX = 64;               // partials summed serially per bucket
-constexpr int HEAVY_FAN = 8;                 // fan-in of the heavy-bucket tree
 
 // ---------------------------------------------------------------- digits
 // Booth-style signed recoding: d_t = v_t + k_{ct-1} - 2^c * k_{ct+c-1}, with
@@ -63,13 +62,34 @@ __global__ void k_to_mont(const uint32_t* __restrict__ in, uint32_t* __restrict_
   }
 }
 
+// ------------------------------------------ block-level hot-key aggregation
+// Skewed scalars (the sparse witness: 40 % of the scalars are 1)
+// send one bucket a large share of all entries.  Warp aggregation leaves one
+// global atomic per warp on that bucket's counter, and same-address atomics
+// serialise in one L2 slice (ncu r01: the sort of the 2^26 sparse MSM spent
+// ~8 ms there).  A warp whose key is shared by >= HOT_MIN lanes therefore adds
+// into a small shared-memory table first (open addressing on the key), and the
+// block issues one global atomic per hot key.
+constexpr int HOT_SLOTS = 32;
+constexpr uint32_t HOT_MIN = 4;
+constexpr uint32_t HOT_EMPTY = 0xffffffffu;
+
+GZ_DEV int hot_slot(uint32_t* s_key, uint32_t key) {
+  int h = (int)((key * 2654435761u) >> 27);            // 5 bits: HOT_SLOTS = 32
+#pragma unroll 1
+  for (int q = 0; q < HOT_SLOTS; ++q, h = (h + 1) & (HOT_SLOTS - 1)) {
+    const uint32_t old = atomicCAS(&s_key[h], HOT_EMPTY, key);
+    if (old == HOT_EMPTY || old == key) return h;
+  }
+  return -1;                                          // table full: global atomic
+}
+
 // ----------------------------------------------- a2 digits + histogram
 // One thread per point.  The block stages its scalars in shared memory
 // (coalesced 16-B loads; [word][thread] layout, conflict-free), each thread
 // derives all W digits, writes the digit codes window-major (codes[t*n + i],
 // coalesced) and counts them into the global bucket histogram with
-// warp-aggregated atomics: lanes holding the same bucket (the sparse witness's
-// hot bucket 1) issue ONE atomic (PAPER.md:243-245 skew).
+// warp-aggregated atomics, block-aggregated for hot keys (above).
 constexpr int DIGIT_THREADS = 256;
 template <class C>
 __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __restrict__ sc, size_t n, int c, int W,
@@ -77,9 +97,11 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
                                                           uint32_t* __restrict__ counts) {
   constexpr int NS = C::NS;
   __shared__ uint32_t s_sc[NS * DIGIT_THREADS];
+  __shared__ uint32_t s_key[HOT_SLOTS], s_cnt[HOT_SLOTS];
   const size_t base = (size_t)blockIdx.x * DIGIT_THREADS;
   const size_t left = n > base ? n - base : 0;
   const int rows = left < (size_t)DIGIT_THREADS ? (int)left : DIGIT_THREADS;
+  if (threadIdx.x < HOT_SLOTS) { s_key[threadIdx.x] = HOT_EMPTY; s_cnt[threadIdx.x] = 0; }
   // coalesced staging: the block's scalars are rows*NS contiguous words
   for (int q = threadIdx.x; q < rows * NS; q += DIGIT_THREADS) {
     const int r = q / NS, w = q % NS;
@@ -97,9 +119,16 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
     if (code) {
       const uint32_t key = (uint32_t)t * key_stride + (code & ~VAL_NEG) - 1u;
       const unsigned peers = __match_any_sync(__activemask(), key);
-      if (lane == __ffs(peers) - 1) atomicAdd(&counts[key], (uint32_t)__popc(peers));
+      if (lane == __ffs(peers) - 1) {
+        const uint32_t cnt = (uint32_t)__popc(peers);
+        const int h = cnt >= HOT_MIN ? hot_slot(s_key, key) : -1;
+        if (h >= 0) atomicAdd(&s_cnt[h], cnt);
+        else atomicAdd(&counts[key], cnt);
+      }
     }
   }
+  __syncthreads();
+  if (tid < HOT_SLOTS && s_key[tid] != HOT_EMPTY) atomicAdd(&counts[s_key[tid]], s_cnt[tid]);
 }
 
 // Cross-window consolidation (§4.1; NEXT-1): with prepared
@@ -111,25 +140,43 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
 // flight write into one or two windows' 4n-byte ranges, which stay resident in
 // L2 until their sectors are complete.  Positions come from the bucket cursors
 // (offsets copy) with warp-aggregated atomics: one atomic per distinct bucket
-// per warp; the order inside a bucket is irrelevant (exact abelian sum,
+// per warp, and one per block for hot keys (the block's run is reserved after
+// a barrier); the order inside a bucket is irrelevant (exact abelian sum,
 // DESIGN.md reading R11).
 constexpr int SCATTER_THREADS = 256;
 static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32_t* __restrict__ codes, size_t n,
                                                              uint32_t bpw, uint32_t key_stride, uint32_t val_stride,
                                                              uint32_t* __restrict__ cursor, uint32_t* __restrict__ vals) {
+  __shared__ uint32_t s_key[HOT_SLOTS], s_cnt[HOT_SLOTS], s_base[HOT_SLOTS];
+  const int tid = threadIdx.x;
+  if (tid < HOT_SLOTS) { s_key[tid] = HOT_EMPTY; s_cnt[tid] = 0; }
+  __syncthreads();
   const uint32_t t = blockIdx.x / bpw;
-  const size_t i = (size_t)(blockIdx.x % bpw) * SCATTER_THREADS + threadIdx.x;
-  if (i >= n) return;
-  const uint32_t code = codes[(size_t)t * n + i];
-  if (!code) return;
+  const size_t i = (size_t)(blockIdx.x % bpw) * SCATTER_THREADS + tid;
+  const uint32_t code = i < n ? codes[(size_t)t * n + i] : 0u;
   const uint32_t key = t * key_stride + (code & ~VAL_NEG) - 1u;
-  const unsigned peers = __match_any_sync(__activemask(), key);
-  const int lane = threadIdx.x & 31;
-  const int leader = __ffs(peers) - 1;
+  const int lane = tid & 31;
+  unsigned peers = 0;
+  int leader = 0, h = -1;
   uint32_t pos = 0;
-  if (lane == leader) pos = atomicAdd(&cursor[key], (uint32_t)__popc(peers));
-  pos = __shfl_sync(peers, pos, leader) + __popc(peers & ((1u << lane) - 1u));
-  vals[pos] = (t * val_stride + (uint32_t)i) | (code & VAL_NEG);
+  if (code) {
+    peers = __match_any_sync(__activemask(), key);
+    leader = __ffs(peers) - 1;
+    if (lane == leader) {
+      const uint32_t cnt = (uint32_t)__popc(peers);
+      h = cnt >= HOT_MIN ? hot_slot(s_key, key) : -1;
+      if (h >= 0) pos = atomicAdd(&s_cnt[h], cnt);          // offset inside the block's run
+      else pos = atomicAdd(&cursor[key], cnt);
+    }
+  }
+  __syncthreads();
+  if (tid < HOT_SLOTS && s_key[tid] != HOT_EMPTY) s_base[tid] = atomicAdd(&cursor[s_key[tid]], s_cnt[tid]);
+  __syncthreads();
+  if (code) {
+    if (lane == leader && h >= 0) pos += s_base[h];
+    pos = __shfl_sync(peers, pos, leader) + __popc(peers & ((1u << lane) - 1u));
+    vals[pos] = (t * val_stride + (uint32_t)i) | (code & VAL_NEG);
+  }
 }
 
 // ----------------------------------------------------- scan (exclusive)
@@ -353,11 +400,13 @@ __global__ void __launch_bounds__(128, AccumCfg<C>::MIN_CTAS)
 // Thread per bucket of the group: a bucket spanning local chunks t0 < t1 has
 // q = t1 - t0 + 1 partials (slot 2*(base+t0)+1, then head slots 2*(base+t)).
 // q <= MERGE_QMAX: summed here.  Larger q (a heavy bucket of a skewed input)
-// raises *heavy and is reduced by the k_heavy_level tree instead.
+// is appended to the group's heavy list (k, t0, t1) and reduced by the
+// k_heavy_* kernels instead.
 template <class C>
 __global__ void __launch_bounds__(128) k_merge_bucket(const uint32_t* __restrict__ off, Group grp, int S,
                                                       const uint32_t* __restrict__ spay, uint32_t* __restrict__ buckets,
-                                                      uint32_t* __restrict__ heavy) {
+                                                      uint32_t* __restrict__ heavy_cnt, uint4* __restrict__ hlist,
+                                                      uint32_t hmax) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
   const uint32_t G0 = __ldg(off + grp.key_lo);
@@ -367,7 +416,11 @@ __global__ void __launch_bounds__(128) k_merge_bucket(const uint32_t* __restrict
     if (b1 == b0) continue;
     const uint32_t t0 = (b0 - G0) / S, t1 = (b1 - 1 - G0) / S;
     if (t0 == t1) continue;                              // written by k_accum
-    if (t1 - t0 + 1 > (uint32_t)MERGE_QMAX) { *heavy = 1u; continue; }
+    if (t1 - t0 + 1 > (uint32_t)MERGE_QMAX) {
+      const uint32_t h = atomicAdd(heavy_cnt, 1u);
+      if (h < hmax) hlist[h] = make_uint4(k, t0, t1, 0u);   // hmax bounds every input (planner)
+      continue;
+    }
     typename EC_::Xyzz acc, X;
     EC_::load(acc, spay + (size_t)(2 * (grp.chunk_base + t0) + 1) * 4 * N);
     for (uint32_t t = t0 + 1; t <= t1; ++t) {
@@ -378,60 +431,96 @@ __global__ void __launch_bounds__(128) k_merge_bucket(const uint32_t* __restrict
   }
 }
 
-// Heavy buckets: in-place tree over their head slots.  Head u (0-based, local
-// chunk t0+1+u) is a level-l leader when u % (stride*FAN) == 0; it absorbs
-// heads u + j*stride, j = 1..FAN-1 (leaders of level l-1).  After
-// ceil(log_FAN q) levels head 0 holds the sum of all heads.
-template <class C>
-__global__ void __launch_bounds__(128) k_heavy_level(const uint32_t* __restrict__ off, Group grp, int S,
-                                                     uint32_t stride, const uint32_t* __restrict__ heavy,
-                                                     uint32_t* __restrict__ spay) {
-  using EC_ = EC<C>;
-  constexpr int N = C::N;
-  if (!*heavy) return;
-  const uint32_t G0 = __ldg(off + grp.key_lo), G1 = __ldg(off + grp.key_hi);
-  const uint32_t nchunks = (G1 - G0 + S - 1) / S;
-  const uint64_t span = (uint64_t)stride * HEAVY_FAN;
-  for (uint32_t t = blockIdx.x * blockDim.x + threadIdx.x; t < nchunks; t += gridDim.x * blockDim.x) {
-    const uint32_t beg = G0 + t * (uint32_t)S;
-    const uint32_t k = find_bucket(off, grp.key_lo, grp.key_hi, beg);
-    const uint32_t b0 = __ldg(off + k), b1 = __ldg(off + k + 1);
-    if (b0 >= beg) continue;                               // chunk t has no head slot
-    const uint32_t t0 = (b0 - G0) / S, t1 = (b1 - 1 - G0) / S;
-    if (t1 - t0 + 1 <= (uint32_t)MERGE_QMAX) continue;     // light bucket
-    const uint32_t u = t - t0 - 1, nheads = t1 - t0;
-    if (u % span) continue;
-    typename EC_::Xyzz acc, X;
-    EC_::load(acc, spay + (size_t)(2 * (grp.chunk_base + t)) * 4 * N);
-    for (uint32_t j = 1; j < (uint32_t)HEAVY_FAN; ++j) {
-      const uint64_t v = u + (uint64_t)j * stride;
-      if (v >= nheads) break;
-      EC_::load(X, spay + (size_t)(2 * (grp.chunk_base + t0 + 1 + v)) * 4 * N);
-      ec_add<C>(acc, X);
-    }
-    EC_::store(spay + (size_t)(2 * (grp.chunk_base + t)) * 4 * N, acc);
+// Heavy buckets: the head slots of chunks t0+1 .. t1 (nheads = t1 - t0) are
+// summed by a tree of fan-in HEAVY_SPAN = 1024 (one CTA of 128 threads, 8
+// serial adds per thread, then a shared-memory tree).  Level l (stride
+// HEAVY_SPAN^l) sums the level-(l-1) results at heads u = m * stride, job
+// (h, seg) covering m in [seg SPAN, (seg+1) SPAN) and writing head seg SPAN
+// stride.  job_off[l][h] = first job of bucket h at level l (k_heavy_plan), so
+// a CTA maps its job to (h, seg) by binary search; no per-chunk bucket lookups.
+constexpr int HEAVY_THREADS = 128;
+constexpr uint32_t HEAVY_SPAN = 1024;
+
+static __global__ void k_heavy_plan(const uint32_t* __restrict__ heavy_cnt, const uint4* __restrict__ hlist,
+                                    uint32_t hmax, int levels, uint32_t* __restrict__ job_off) {
+  // one block: job_off[l * (hmax + 1) + h], exclusive prefix over h (serial
+  // per level on thread l: the heavy list is short -- usually 1 .. W entries)
+  const uint32_t H = min(*heavy_cnt, hmax);
+  const int l = threadIdx.x;
+  if (l >= levels) return;
+  uint64_t stride = 1;
+  for (int q = 0; q < l; ++q) stride *= HEAVY_SPAN;
+  uint32_t acc = 0;
+  uint32_t* jo = job_off + (size_t)l * (hmax + 1);
+  for (uint32_t h = 0; h < H; ++h) {
+    jo[h] = acc;
+    const uint4 e = hlist[h];
+    const uint64_t nheads = e.z - e.y;
+    const uint64_t m = (nheads + stride - 1) / stride;           // heads alive at this level
+    acc += m > 1 ? (uint32_t)((m + HEAVY_SPAN - 1) / HEAVY_SPAN) : 0u;
   }
+  jo[H] = acc;
 }
 
 template <class C>
-__global__ void __launch_bounds__(128) k_heavy_final(const uint32_t* __restrict__ off, Group grp, int S,
-                                                     const uint32_t* __restrict__ heavy,
+__global__ void __launch_bounds__(HEAVY_THREADS) k_heavy_tree(const uint32_t* __restrict__ heavy_cnt,
+                                                              const uint4* __restrict__ hlist, uint32_t hmax,
+                                                              const uint32_t* __restrict__ job_off, uint64_t stride,
+                                                              Group grp, uint32_t* __restrict__ spay) {
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  extern __shared__ __align__(16) uint32_t heavy_smem[];
+  const uint32_t H = min(*heavy_cnt, hmax);
+  const uint32_t jobs = job_off[H];
+  for (uint32_t job = blockIdx.x; job < jobs; job += gridDim.x) {
+    uint32_t lo = 0, hi = H;                 // largest h with job_off[h] <= job
+    while (hi - lo > 1) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (job_off[mid] <= job) lo = mid; else hi = mid;
+    }
+    const uint4 e = hlist[lo];
+    const uint32_t t0 = e.y;
+    const uint64_t nheads = e.z - e.y;
+    const uint64_t alive = (nheads + stride - 1) / stride;
+    const uint64_t m0 = (uint64_t)(job - job_off[lo]) * HEAVY_SPAN;
+    const uint64_t m1 = alive < m0 + HEAVY_SPAN ? alive : m0 + HEAVY_SPAN;
+    auto slot = [&](uint64_t m) { return spay + (size_t)(2 * (grp.chunk_base + t0 + 1 + m * stride)) * 4 * N; };
+    typename EC_::Xyzz acc, X;
+    EC_::set_inf(acc);
+    for (uint64_t m = m0 + threadIdx.x; m < m1; m += HEAVY_THREADS) {
+      EC_::load(X, slot(m));
+      ec_add_hot<C>(acc, X);
+    }
+    EC_::store(heavy_smem + threadIdx.x * 4 * N, acc);
+    __syncthreads();
+    for (int w = HEAVY_THREADS / 2; w > 0; w >>= 1) {
+      if (threadIdx.x < w) {
+        EC_::load(X, heavy_smem + (threadIdx.x + w) * 4 * N);
+        ec_add_hot<C>(acc, X);
+        EC_::store(heavy_smem + threadIdx.x * 4 * N, acc);
+      }
+      __syncthreads();
+    }
+    if (threadIdx.x == 0) EC_::store(slot(m0), acc);
+    __syncthreads();
+  }
+}
+
+// bucket k = tail partial of chunk t0 + the summed heads (head of chunk t0+1)
+template <class C>
+__global__ void __launch_bounds__(128) k_heavy_final(const uint32_t* __restrict__ heavy_cnt,
+                                                     const uint4* __restrict__ hlist, uint32_t hmax, Group grp,
                                                      const uint32_t* __restrict__ spay, uint32_t* __restrict__ buckets) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
-  if (!*heavy) return;
-  const uint32_t G0 = __ldg(off + grp.key_lo);
-  for (uint32_t k = grp.key_lo + blockIdx.x * blockDim.x + threadIdx.x; k < grp.key_hi;
-       k += gridDim.x * blockDim.x) {
-    const uint32_t b0 = __ldg(off + k), b1 = __ldg(off + k + 1);
-    if (b1 == b0) continue;
-    const uint32_t t0 = (b0 - G0) / S, t1 = (b1 - 1 - G0) / S;
-    if (t1 - t0 + 1 <= (uint32_t)MERGE_QMAX) continue;
+  const uint32_t H = min(*heavy_cnt, hmax);
+  for (uint32_t h = blockIdx.x * blockDim.x + threadIdx.x; h < H; h += gridDim.x * blockDim.x) {
+    const uint4 e = hlist[h];
     typename EC_::Xyzz acc, X;
-    EC_::load(acc, spay + (size_t)(2 * (grp.chunk_base + t0) + 1) * 4 * N);
-    EC_::load(X, spay + (size_t)(2 * (grp.chunk_base + t0 + 1)) * 4 * N);
+    EC_::load(acc, spay + (size_t)(2 * (grp.chunk_base + e.y) + 1) * 4 * N);
+    EC_::load(X, spay + (size_t)(2 * (grp.chunk_base + e.y + 1)) * 4 * N);
     ec_add<C>(acc, X);
-    EC_::store(buckets + (size_t)k * 4 * N, acc);
+    EC_::store(buckets + (size_t)e.x * 4 * N, acc);
   }
 }
 

@@ -238,3 +238,23 @@ def test_weighted_default_and_unweighted_prepare():
     h2 = gz.PreparedPoints(curve, dev(pts), weighted=False)
     assert not h2.info()["weighted"]
     assert np.array_equal(host(h2.msm(dev(k))), want)
+
+
+@pytest.mark.parametrize("curve", ["bn254", "bls12_381"])
+def test_heavy_buckets_tree(curve):
+    """Skew beyond MERGE_QMAX chunks per bucket: the heavy-list tree (fan-in
+    1024, several levels with chunk size 1) against the oracle's closed form.
+    all-equal scalars put every point of every window into ONE bucket per
+    window (W heavy buckets); all-one scalars make one bucket of n entries."""
+    gz = require_cuda()
+    n = 1 << 13
+    pts, d = oracle_points(curve, n)
+    c = curves.get(curve)
+    k_eq = np.tile(synth.scalars(curve, 1, 4242), (n, 1))
+    k_one = synth.scalars(curve, n, 1, "all_one")
+    for k in (k_eq, k_one):
+        want = oracle.closed_form(curve, k, d)
+        for chunk in (0, 1, 7):
+            gz.set_config(0, chunk)
+            assert np.array_equal(run(gz, curve, pts, k), want), chunk
+    gz.set_config(0, 0)
