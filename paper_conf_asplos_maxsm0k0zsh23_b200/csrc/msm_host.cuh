@@ -209,11 +209,13 @@ struct Impl {
     return per_sm * device_sm_count();
   }
 
-  static gzkp_status to_mont(const void* in, void* out, size_t n, cudaStream_t s) {
+  static gzkp_status to_mont(const void* in, void* out, size_t n, cudaStream_t s) { return to_mont_sc(in, out, n, nullptr, s); }
+  static gzkp_status to_mont_sc(const void* in, void* out, size_t n, const void* sc, cudaStream_t s) {
     if (!n) return GZKP_SUCCESS;
     const int threads = 256;
-    const int grid = (int)std::min<size_t>((n + threads - 1) / threads, (size_t)device_sm_count() * 16);
-    k_to_mont<C><<<grid, threads, 0, s>>>((const uint32_t*)in, (uint32_t*)out, n);
+    const size_t tiles = (n + 255) / 256;                    // one 256-point tile per warp
+    const int grid = (int)std::min<size_t>((tiles + 7) / 8, (size_t)device_sm_count() * 16);
+    k_to_mont<C><<<grid, threads, 0, s>>>((const uint32_t*)in, (uint32_t*)out, n, (const uint32_t*)sc);
     GZ_CHECK(cudaGetLastError());
     return GZKP_SUCCESS;
   }
@@ -254,7 +256,7 @@ struct Impl {
     // a1: points -> Montgomery (skipped for prepared handles)
     const uint32_t* pts = (const uint32_t*)call.points;
     if (!call.prepared) {
-      if (gzkp_status st = to_mont(call.points, U(p.o_pts), n, s)) return st;
+      if (gzkp_status st = to_mont_sc(call.points, U(p.o_pts), n, call.scalars, s)) return st;
       pts = U(p.o_pts);
       ++launches;
     }
@@ -272,7 +274,8 @@ struct Impl {
     k_scan_top<<<1, SCAN_THREADS, 0, s>>>(U(p.o_tiles), ntiles, U(p.o_offsets) + p.M);
     k_scan_add<<<ntiles, SCAN_THREADS, 0, s>>>(U(p.o_offsets), U(p.o_cursor), p.M, U(p.o_tiles));
     // a3: scatter into bucket order (window-major grid)
-    k_scatter<<<(unsigned)((uint64_t)bpw * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw, key_stride,
+    const uint32_t bpw_s = (uint32_t)((n + SCATTER_TILE - 1) / SCATTER_TILE);
+    k_scatter<<<(unsigned)((uint64_t)bpw_s * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw_s, key_stride,
                                                                          p.val_stride, U(p.o_cursor), U(p.o_vals));
     GZ_CHECK(cudaGetLastError());
     launches += 5;

@@ -47,18 +47,49 @@ GZ_DEV uint32_t digit_code(int d) { return d ? ((uint32_t)abs(d) | (d < 0 ? VAL_
 
 // ------------------------------------------------------------ a1 to_mont
 template <class C>
-__global__ void k_to_mont(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, size_t n) {
+__global__ void __launch_bounds__(256) k_to_mont(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, size_t n,
+                                                 const uint32_t* __restrict__ sc) {
+  // sc (optional): the call's scalars.  A point whose scalar is 0 is never
+  // gathered by the accumulation, so its conversion is skipped (half the
+  // points of the sparse witness; the conversion is IMAD-bound).
+  // Each warp compacts the non-zero points of a 256-point tile into a shared
+  // list first, so the products run on full warps instead of diverged ones.
   using Fp = Field<C>;
   using E = EC<C>;
   constexpr int N = C::N;
-  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
-    uint32_t x[N], y[N];
-    E::ld(x, in + i * 2 * N);
-    E::ld(y, in + i * 2 * N + N);
-    Fp::to_mont(x, x);
-    Fp::to_mont(y, y);
-    E::st(out + i * 2 * N, x);
-    E::st(out + i * 2 * N + N, y);
+  constexpr int TILE = 256;
+  __shared__ uint32_t s_list[8][TILE];
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint32_t* list = s_list[warp & 7];
+  const size_t wid = (blockIdx.x * (size_t)blockDim.x + threadIdx.x) >> 5;
+  const size_t nwarps = ((size_t)gridDim.x * blockDim.x) >> 5;
+  for (size_t base = wid * TILE; base < n; base += nwarps * TILE) {
+    int cnt = 0;
+    for (int q = 0; q < TILE; q += 32) {
+      const size_t i = base + q + lane;
+      bool live = i < n;
+      if (live && sc) {
+        uint32_t any = 0;
+#pragma unroll
+        for (int w = 0; w < C::NS; ++w) any |= __ldg(sc + i * C::NS + w);
+        live = any != 0;
+      }
+      const unsigned m = __ballot_sync(0xffffffffu, live);
+      if (live) list[cnt + __popc(m & ((1u << lane) - 1u))] = (uint32_t)(q + lane);
+      cnt += __popc(m);
+    }
+    __syncwarp();
+    for (int e = lane; e < cnt; e += 32) {
+      const size_t i = base + list[e];
+      uint32_t x[N], y[N];
+      E::ld(x, in + i * 2 * N);
+      E::ld(y, in + i * 2 * N + N);
+      Fp::to_mont(x, x);
+      Fp::to_mont(y, y);
+      E::st(out + i * 2 * N, x);
+      E::st(out + i * 2 * N + N, y);
+    }
+    __syncwarp();
   }
 }
 
@@ -144,6 +175,8 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
 // a barrier); the order inside a bucket is irrelevant (exact abelian sum,
 // DESIGN.md reading R11).
 constexpr int SCATTER_THREADS = 256;
+constexpr int SCATTER_PER_THREAD = 4;        // consecutive points of one window per thread (one 16-B load)
+constexpr int SCATTER_TILE = SCATTER_THREADS * SCATTER_PER_THREAD;
 static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32_t* __restrict__ codes, size_t n,
                                                              uint32_t bpw, uint32_t key_stride, uint32_t val_stride,
                                                              uint32_t* __restrict__ cursor, uint32_t* __restrict__ vals) {
@@ -152,30 +185,47 @@ static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32
   if (tid < HOT_SLOTS) { s_key[tid] = HOT_EMPTY; s_cnt[tid] = 0; }
   __syncthreads();
   const uint32_t t = blockIdx.x / bpw;
-  const size_t i = (size_t)(blockIdx.x % bpw) * SCATTER_THREADS + tid;
-  const uint32_t code = i < n ? codes[(size_t)t * n + i] : 0u;
-  const uint32_t key = t * key_stride + (code & ~VAL_NEG) - 1u;
+  const size_t i0 = (size_t)(blockIdx.x % bpw) * SCATTER_TILE + (size_t)tid * SCATTER_PER_THREAD;
+  const uint32_t* crow = codes + (size_t)t * n;
+  uint32_t code[SCATTER_PER_THREAD];
+  if (i0 + SCATTER_PER_THREAD <= n && (n % 4) == 0) {
+    const uint4 v = *reinterpret_cast<const uint4*>(crow + i0);
+    code[0] = v.x; code[1] = v.y; code[2] = v.z; code[3] = v.w;
+  } else {
+#pragma unroll
+    for (int q = 0; q < SCATTER_PER_THREAD; ++q) code[q] = i0 + q < n ? crow[i0 + q] : 0u;
+  }
   const int lane = tid & 31;
-  unsigned peers = 0;
-  int leader = 0, h = -1;
-  uint32_t pos = 0;
-  if (code) {
-    peers = __match_any_sync(__activemask(), key);
-    leader = __ffs(peers) - 1;
-    if (lane == leader) {
-      const uint32_t cnt = (uint32_t)__popc(peers);
-      h = cnt >= HOT_MIN ? hot_slot(s_key, key) : -1;
-      if (h >= 0) pos = atomicAdd(&s_cnt[h], cnt);          // offset inside the block's run
-      else pos = atomicAdd(&cursor[key], cnt);
+  unsigned peers[SCATTER_PER_THREAD];
+  int leader[SCATTER_PER_THREAD], h[SCATTER_PER_THREAD];
+  uint32_t pos[SCATTER_PER_THREAD];
+#pragma unroll
+  for (int q = 0; q < SCATTER_PER_THREAD; ++q) {
+    peers[q] = 0; leader[q] = 0; h[q] = -1; pos[q] = 0;
+    const uint32_t key = t * key_stride + (code[q] & ~VAL_NEG) - 1u;
+    if (!__any_sync(0xffffffffu, code[q] != 0)) continue;        // sparse windows: mostly empty
+    if (code[q]) {
+      peers[q] = __match_any_sync(__activemask(), key);
+      leader[q] = __ffs(peers[q]) - 1;
+      if (lane == leader[q]) {
+        const uint32_t cnt = (uint32_t)__popc(peers[q]);
+        h[q] = cnt >= HOT_MIN ? hot_slot(s_key, key) : -1;
+        if (h[q] >= 0) pos[q] = atomicAdd(&s_cnt[h[q]], cnt);     // offset inside the block's run
+        else pos[q] = atomicAdd(&cursor[key], cnt);
+      }
     }
   }
   __syncthreads();
   if (tid < HOT_SLOTS && s_key[tid] != HOT_EMPTY) s_base[tid] = atomicAdd(&cursor[s_key[tid]], s_cnt[tid]);
   __syncthreads();
-  if (code) {
-    if (lane == leader && h >= 0) pos += s_base[h];
-    pos = __shfl_sync(peers, pos, leader) + __popc(peers & ((1u << lane) - 1u));
-    vals[pos] = (t * val_stride + (uint32_t)i) | (code & VAL_NEG);
+#pragma unroll
+  for (int q = 0; q < SCATTER_PER_THREAD; ++q) {
+    if (code[q]) {
+      uint32_t p = pos[q];
+      if (lane == leader[q] && h[q] >= 0) p += s_base[h[q]];
+      p = __shfl_sync(peers[q], p, leader[q]) + __popc(peers[q] & ((1u << lane) - 1u));
+      vals[p] = (t * val_stride + (uint32_t)(i0 + q)) | (code[q] & VAL_NEG);
+    }
   }
 }
 
