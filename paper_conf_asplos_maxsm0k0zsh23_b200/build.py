@@ -64,10 +64,11 @@ def _compile(src: str, verbose: bool) -> str:
 
 
 def build(force: bool = False, verbose: bool = False) -> str:
+    """Recompile each translation unit whose object is older than the source or
+    any header in its depfile (headers edited while a build runs are caught:
+    the check is per object, never "library newer than the sources"), then
+    relink if any object is newer than the library."""
     srcs = _sources()
-    deps = srcs + _headers()
-    if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= _newest(deps):
-        return LIB
     os.makedirs(BUILD, exist_ok=True)
     todo = []
     objs = []
@@ -76,8 +77,11 @@ def build(force: bool = False, verbose: bool = False) -> str:
         objs.append(obj)
         if force or verbose or not os.path.exists(obj) or os.path.getmtime(obj) < _newest(_deps(obj, s)):
             todo.append(s)
-    with cf.ThreadPoolExecutor(max_workers=max(1, min(len(todo), os.cpu_count() or 4))) as ex:
-        list(ex.map(lambda s: _compile(s, verbose), todo))
+    if todo:
+        with cf.ThreadPoolExecutor(max_workers=max(1, min(len(todo), os.cpu_count() or 4))) as ex:
+            list(ex.map(lambda s: _compile(s, verbose), todo))
+    if not todo and os.path.exists(LIB) and os.path.getmtime(LIB) >= _newest(objs):
+        return LIB
     tmp = LIB + ".tmp.%d" % os.getpid()
     cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart", "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)

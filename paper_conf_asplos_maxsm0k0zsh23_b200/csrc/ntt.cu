@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <map>
 #include <mutex>
 #include <tuple>
@@ -70,8 +71,16 @@ struct NttImpl {
     if (gzkp_status st = tables(fid, log_n, inverse, s, &tb)) return st;
     static bool attr = false;
     const size_t smem = ((size_t)1 << TILE_LOG) * L * 4;
+    // register budget: MIN_CTAS CTAs/SM (the shared-memory limit) or, with
+    // GZKP_NTT_MINB=2 (8-limb fields), 2 CTAs/SM with up to 128 registers
+    static const bool two = [] {
+      const char* e = getenv("GZKP_NTT_MINB");
+      return L <= 8 && e && atoi(e) == 2;
+    }();
+    auto kern = two ? k_ntt_pass<R, 2> : k_ntt_pass<R>;
     if (!attr) {
       NTT_CHECK(cudaFuncSetAttribute(k_ntt_pass<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+      NTT_CHECK(cudaFuncSetAttribute(k_ntt_pass<R, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
       attr = true;
     }
     *launches = 0;
@@ -99,8 +108,7 @@ struct NttImpl {
       uint32_t* dst = last ? (uint32_t*)out : (uint32_t*)ws;
       const int flags = (p == 0 ? NTT_FIRST : 0) | (last ? NTT_LAST : 0) | (last && inverse ? NTT_SCALE : 0);
       const size_t sm = ((size_t)1 << (nb + logG)) * L * 4;
-      k_ntt_pass<R><<<grid, NTT_THREADS, sm, s>>>(src, dst, tb->tw, log_n, t0, nb, logG, flags,
-                                                  tb->tw + tb->half * L);
+      kern<<<grid, NTT_THREADS, sm, s>>>(src, dst, tb->tw, log_n, t0, nb, logG, flags, tb->tw + tb->half * L);
       NTT_CHECK(cudaGetLastError());
       ++*launches;
       src = dst;

@@ -111,8 +111,8 @@ GZ_DEV void sm_st(uint32_t* sm, int slot, const uint32_t d[R::N]) {
 // of the tile (j < 2^nb, g < G) is x[hi 2^(s+nb) + j 2^s + lo] with
 // q = q0 + g, kept at shared slot j G + g.
 // tw[k] = w^k (Montgomery), k < N/2 (w = w_N, or w_N^-1 for the inverse).
-template <class R>
-__global__ void __launch_bounds__(NTT_THREADS, NttCfg<R>::MIN_CTAS) k_ntt_pass(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst,
+template <class R, int MINB = NttCfg<R>::MIN_CTAS>
+__global__ void __launch_bounds__(NTT_THREADS, MINB) k_ntt_pass(const uint32_t* __restrict__ src, uint32_t* __restrict__ dst,
                                                           const uint32_t* __restrict__ tw, int log_n, int t0, int nb,
                                                           int logG, int flags, const uint32_t* __restrict__ scale) {
   using Fr = F<R>;
