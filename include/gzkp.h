@@ -148,6 +148,11 @@ gzkp_status gzkp_comm_destroy(void *comm);
  * exchanged with ONE ncclAllGather, and every rank writes the same `out`. */
 gzkp_status gzkp_msm_sharded(int curve, const void *points_affine, const void *scalars,
                              size_t n_local, void *out, gzkp_stream stream, void *comm);
+/* Same collective on prepared points: every rank passes the handle of ITS
+ * shard (gzkp_points_prepare on the local slice; weighted tables remove the
+ * per-rank window combination) and its n_local <= prepared count scalars. */
+gzkp_status gzkp_msm_prepared_sharded(const void *handle, const void *scalars, size_t n_local, void *out,
+                                      gzkp_stream stream, void *comm);
 
 /* --- NTT over the scalar field F_r -------------------
  * The POLY stage of the prover (§2.2, §3): for N = 2^log_n and

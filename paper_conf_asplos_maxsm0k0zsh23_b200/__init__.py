@@ -66,6 +66,7 @@ def lib():
             "gzkp_comm_init": ([i32, i32, ctypes.c_char_p, ctypes.POINTER(vp)], i32),
             "gzkp_comm_destroy": ([vp], i32),
             "gzkp_msm_sharded": ([i32, vp, vp, sz, vp, vp, vp], i32),
+            "gzkp_msm_prepared_sharded": ([vp, vp, sz, vp, vp, vp], i32),
             "gzkp_fixed_base_mul": ([i32, vp, sz, vp, vp], i32),
             "gzkp_field_op": ([i32, i32, vp, vp, vp, sz, vp], i32),
             "gzkp_ec_op": ([i32, i32, vp, vp, vp, sz, vp], i32),
@@ -425,7 +426,19 @@ def msm_sharded(curve, points_local, scalars_local, comm: Comm, out=None, stream
     return out
 
 
+def msm_prepared_sharded(prepared: "PreparedPoints", scalars_local, comm: Comm, out=None, stream=None):
+    """Collective MSM over per-rank prepared shards (one all-gather)."""
+    torch = _torch()
+    L, Ls = field_limbs(prepared.curve), scalar_limbs(prepared.curve)
+    K = _dev_u32(scalars_local, Ls, "scalars")
+    if out is None:
+        out = torch.empty(2 * L, dtype=torch.int32, device=K.device)
+    _check(lib().gzkp_msm_prepared_sharded(prepared.handle, K.data_ptr(), K.shape[0], out.data_ptr(),
+                                           _stream_ptr(stream), comm.handle), "gzkp_msm_prepared_sharded")
+    return out
+
+
 __all__ = ["CURVES", "GzkpError", "lib", "msm", "msm_host", "PreparedPoints", "msm_partial", "combine_partials",
-           "fixed_base_mul", "field_op", "ec_op", "Comm", "msm_sharded", "shard_range", "set_config",
+           "fixed_base_mul", "field_op", "ec_op", "Comm", "msm_sharded", "msm_prepared_sharded", "shard_range", "set_config",
            "window_bits", "workspace_bytes", "set_profiling", "profile_read", "field_limbs", "scalar_limbs", "to_device",
            "to_numpy", "ntt", "ntt_max_log", "ntt_last_launches", "scalar_field_op"]

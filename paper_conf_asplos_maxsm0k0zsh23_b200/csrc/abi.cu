@@ -424,12 +424,13 @@ gzkp_status gzkp_prepared_info(const void* handle, int* window_bits, int* window
   return GZKP_SUCCESS;
 }
 
-gzkp_status gzkp_msm_prepared(const void* handle, const void* scalars, size_t n, void* out, gzkp_stream stream) {
+static gzkp_status msm_prepared_impl(const void* handle, const void* scalars, size_t n, void* out_affine,
+                                     void* out_partial, gzkp_stream stream) {
   const Prepared* h = (const Prepared*)handle;
   if (!h) return set_error(GZKP_ERROR_INVALID_VALUE, "NULL handle");
   if (n > h->n) return set_error(GZKP_ERROR_INVALID_VALUE, "n exceeds prepared point count");
   const CurveImpl* c = impl_for(h->curve);
-  if (gzkp_status st = check_args(c, h->pts, scalars, n, out)) return st;
+  if (gzkp_status st = check_args(c, h->pts, scalars, n, out_affine ? out_affine : out_partial)) return st;
   init_pool_once();
   MsmCall call;
   call.points = h->pts;
@@ -439,9 +440,14 @@ gzkp_status gzkp_msm_prepared(const void* handle, const void* scalars, size_t n,
   call.table_n = h->n;
   call.scalars = scalars;
   call.n = n;
-  call.out_affine = out;
+  call.out_affine = out_affine;
+  call.out_partial = out_partial;
   call.stream = (cudaStream_t)stream;
   return c->msm(call);
+}
+
+gzkp_status gzkp_msm_prepared(const void* handle, const void* scalars, size_t n, void* out, gzkp_stream stream) {
+  return msm_prepared_impl(handle, scalars, n, out, nullptr, stream);
 }
 
 gzkp_status gzkp_msm_prepared_host(const void* handle, const void* scalars_host, size_t n, void* out_host,
@@ -602,6 +608,25 @@ gzkp_status gzkp_msm_sharded(int curve, const void* points_affine, const void* s
   if (gzkp_status st = nccl_status(nccl().AllGather(cm->partial, cm->gathered, pb, ncclUint8_, cm->comm, s), "ncclAllGather"))
     return st;
   // 3. fold in rank order + normalise; identical bytes on every rank
+  return c->combine(cm->gathered, cm->world, out, s);
+}
+
+/* Sharded MSM on prepared points: each rank prepared ITS shard of the point
+ * vector (gzkp_points_prepare on the local slice, e.g. with the weighted
+ * table), so the per-rank Pippenger has no window combination; the partials
+ * meet in the same single all-gather. */
+gzkp_status gzkp_msm_prepared_sharded(const void* handle, const void* scalars, size_t n_local, void* out,
+                                      gzkp_stream stream, void* comm) {
+  Comm* cm = (Comm*)comm;
+  const Prepared* h = (const Prepared*)handle;
+  if (!cm || !h) return set_error(GZKP_ERROR_INVALID_VALUE, "NULL comm or handle");
+  const CurveImpl* c = impl_for(h->curve);
+  if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
+  cudaStream_t s = (cudaStream_t)stream;
+  if (gzkp_status st = msm_prepared_impl(handle, scalars, n_local, nullptr, cm->partial, stream)) return st;
+  const size_t pb = gzkp_partial_bytes(h->curve);
+  if (gzkp_status st = nccl_status(nccl().AllGather(cm->partial, cm->gathered, pb, ncclUint8_, cm->comm, s), "ncclAllGather"))
+    return st;
   return c->combine(cm->gathered, cm->world, out, s);
 }
 

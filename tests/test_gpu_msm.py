@@ -196,7 +196,12 @@ def test_sharded_single_rank_nccl():
         pts, _ = oracle_points(curve, 1024)
         k = synth.scalars(curve, 1024, 21)
         got = host(gz.msm_sharded(curve, dev(pts), dev(k), comm))
-        assert np.array_equal(got, oracle_msm_cached(curve, pts, k))
+        want = oracle_msm_cached(curve, pts, k)
+        assert np.array_equal(got, want)
+        for weighted in (True, False):                 # prepared shards, same all-gather
+            h = gz.PreparedPoints(curve, dev(pts), weighted=weighted)
+            assert np.array_equal(host(gz.msm_prepared_sharded(h, dev(k), comm)), want)
+            h.release()
         comm.destroy()
     finally:
         dist.destroy_process_group()
