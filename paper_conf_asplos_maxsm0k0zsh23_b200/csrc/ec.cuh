@@ -70,9 +70,8 @@ struct EC {
     Fp::sub(t, t, S);
     Fp::sub(R.X, t, S);                 // X3 = M^2 - 2S
     Fp::sub(t, S, R.X);
-    Fp::mul(t, M, t);
-    Fp::mul(S, W, y);
-    Fp::sub(R.Y, t, S);                 // Y3 = M(S - X3) - W y
+    Fp::neg(S, y);
+    Fp::mul_sum(R.Y, M, t, W, S);       // Y3 = M(S - X3) - W y (one reduction)
     Fp::copy(R.ZZ, V);
     Fp::copy(R.ZZZ, W);
   }
@@ -89,9 +88,8 @@ struct EC {
     Fp::sub(t, t, S);
     Fp::sub(P.X, t, S);                 // X3 = M^2 - 2S
     Fp::sub(t, S, P.X);
-    Fp::mul(t, M, t);
-    Fp::mul(S, W, P.Y);
-    Fp::sub(P.Y, t, S);                 // Y3 = M(S - X3) - W Y1
+    Fp::neg(S, P.Y);
+    Fp::mul_sum(P.Y, M, t, W, S);       // Y3 = M(S - X3) - W Y1 (one reduction)
     Fp::mul(P.ZZ, V, P.ZZ);
     Fp::mul(P.ZZZ, W, P.ZZZ);
   }
@@ -118,9 +116,8 @@ struct EC {
     Fp::sub(t, t, PP);
     Fp::sub(A.X, t, PP);                // X3 = R^2 - PPP - 2Q
     Fp::sub(t, PP, A.X);
-    Fp::mul(t, R, t);
-    Fp::mul(PPP, A.Y, PPP);
-    Fp::sub(A.Y, t, PPP);               // Y3 = R(Q - X3) - Y1 PPP
+    Fp::neg(PP, A.Y);
+    Fp::mul_sum(A.Y, R, t, PP, PPP);    // Y3 = R(Q - X3) - Y1 PPP (one reduction)
   }
 
   // madd_nz with 4 of its 10 products on the FP64 pipe (Dfp<C>::mul, NEXT-2):
@@ -182,9 +179,8 @@ struct EC {
     Fp::sub(t, t, PP);
     Fp::sub(A.X, t, PP);                // X3 = R^2 - PPP - 2Q
     Fp::sub(t, PP, A.X);
-    Fp::mul(t, R, t);
-    Fp::mul(PPP, S1, PPP);
-    Fp::sub(A.Y, t, PPP);               // Y3 = R(Q - X3) - S1 PPP
+    Fp::neg(S1, S1);
+    Fp::mul_sum(A.Y, R, t, S1, PPP);    // Y3 = R(Q - X3) - S1 PPP (one reduction)
   }
 
   // XYZZ (Montgomery) -> canonical affine, O -> (0,0).

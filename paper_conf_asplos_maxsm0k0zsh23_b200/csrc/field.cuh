@@ -360,6 +360,33 @@ struct F {
     ADDC(z[2 * H - 1], EV[2 * H - 1], OD[2 * H - 1]);
   }
 
+  // ---- sum of two Montgomery products with ONE reduction:
+  //   r = (a b + c d) R^-1 mod p.
+  // Both 2N-limb products (prod<N>, 2 N^2 IMAD each) are added, then one SOS
+  // reduction (N (2N + 1)): 876 IMAD for N = 12 instead of 2 x 588.  The
+  // group law's Y3 = R (Q - X3) - Y1 PPP is such a sum (with -Y1 = p - Y1).
+  // Bound: a, b, c, d < p gives T < 2 p^2 < p R (p < R / 2 for every curve
+  // here), which is sos_reduce's precondition (result < 2p, one subtraction).
+  // N >= 24 (MNT4-753) keeps its out-of-line products.
+  GZ_DEV static void mul_sum(uint32_t r[N], const uint32_t a[N], const uint32_t b[N], const uint32_t c[N],
+                             const uint32_t d[N]) {
+    if constexpr (N >= 24) {
+      uint32_t t[N];
+      mul(t, c, d);
+      mul(r, a, b);
+      add(r, r, t);
+    } else {
+      uint32_t T[2 * N], U[2 * N];
+      prod<N>(T, a, b);
+      prod<N>(U, c, d);
+      ADD_CC(T[0], T[0], U[0]);
+#pragma unroll
+      for (int k = 1; k < 2 * N - 1; ++k) ADDC_CC(T[k], T[k], U[k]);
+      ADDC(T[2 * N - 1], T[2 * N - 1], U[2 * N - 1]);
+      sos_reduce(r, T);
+    }
+  }
+
   // ---- Montgomery product with a one-level Karatsuba product (H = N/2):
   //   a b = z0 + z1 2^(32H) + z2 2^(64H),  z0 = a0 b0,  z2 = a1 b1,
   //   z1 = (a0 + a1)(b0 + b1) - z0 - z2 = a0 b1 + a1 b0  (2H + 1 limbs),

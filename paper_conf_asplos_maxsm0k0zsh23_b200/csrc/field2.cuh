@@ -76,6 +76,14 @@ struct F2 {
     Fp::sub(r + NB, sa, t1);
   }
   GZ_DEV static void mul_inline(uint32_t r[N], const uint32_t a[N], const uint32_t b[N]) { mul(r, a, b); }
+  // r = a b + c d (no shared reduction over F_p^2: two Karatsuba products)
+  GZ_DEV static void mul_sum(uint32_t r[N], const uint32_t a[N], const uint32_t b[N], const uint32_t c[N],
+                             const uint32_t d[N]) {
+    uint32_t t[N];
+    mul(t, c, d);
+    mul(r, a, b);
+    add(r, r, t);
+  }
 
   GZ_DEV static void sqr(uint32_t r[N], const uint32_t a[N]) {
     uint32_t s[NB], d[NB], m[NB];

@@ -35,7 +35,8 @@ struct Plan {
   uint64_t E_max = 0, chunks_max = 0;
   // workspace byte offsets
   size_t o_pts = 0, o_codes = 0, o_counts = 0, o_offsets = 0, o_cursor = 0, o_tiles = 0, o_vals = 0,
-         o_spay = 0, o_heavy = 0, o_hlist = 0, o_hjobs = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_win = 0, total = 0;
+         o_spay = 0, o_heavy = 0, o_hlist = 0, o_hjobs = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_terms = 0, o_win = 0, total = 0;
+  size_t seg_stride = 0;  // points between segT and segR in o_seg
   struct Grp {
     int t_lo, t_hi;             // windows (inclusive)
     uint32_t key_lo, key_hi;    // bucket keys
@@ -47,7 +48,7 @@ struct Plan {
   std::vector<Grp> groups;
 };
 
-constexpr uint32_t WIN_PER_BLOCK = 1024;   // segment partials summed per block (stage A)
+inline int ilog2_u64(uint64_t v) { int r = 0; while (v > 1) { v >>= 1; ++r; } return r; }
 
 template <class C>
 struct Impl {
@@ -149,7 +150,7 @@ struct Impl {
     }
     p.chunks_max = 0;
     p.heavy_levels = 0;
-    uint64_t seg_elems = 1, mid_elems = 1, hlist_elems = 0;
+    uint64_t seg_elems = 1, mid_elems = 1, terms_elems = 1, hlist_elems = 0;
     for (auto& g : p.groups) {
       const uint64_t wins = consolidated ? (uint64_t)p.W : (uint64_t)(g.t_hi - g.t_lo + 1);
       const uint64_t bwins = consolidated ? 1 : wins;
@@ -164,7 +165,9 @@ struct Impl {
       g.seg = (int)std::min<uint64_t>(seg, p.B);
       const uint64_t gsegs = p.B / g.seg;
       seg_elems = std::max<uint64_t>(seg_elems, bwins * gsegs);
-      mid_elems = std::max<uint64_t>(mid_elems, bwins * ((gsegs + WIN_PER_BLOCK - 1) / WIN_PER_BLOCK));
+      const uint64_t nb_bits = (uint64_t)ilog2_u64(gsegs) + 1;           // NB + 1 sets
+      mid_elems = std::max<uint64_t>(mid_elems, bwins * nb_bits * ((gsegs + RB_PER - 1) / RB_PER));
+      terms_elems = std::max<uint64_t>(terms_elems, bwins * nb_bits);
       g.chunk_base = p.chunks_max;
       g.chunks_max = (n * wins + p.S - 1) / p.S + 1;
       // a heavy bucket spans > MERGE_QMAX chunks: at most chunks / MERGE_QMAX of them
@@ -193,8 +196,10 @@ struct Impl {
     p.o_state = take(4 * N * 4);
     p.o_buckets = take((size_t)p.M * 4 * N * 4);
     (void)G;
-    p.o_seg = take((size_t)seg_elems * 4 * N * 4);
+    p.seg_stride = (size_t)seg_elems * 4 * N;
+    p.o_seg = take(2 * (size_t)seg_elems * 4 * N * 4);
     p.o_mid = take((size_t)mid_elems * 4 * N * 4);
+    p.o_terms = take((size_t)terms_elems * 4 * N * 4);
     p.o_win = take((size_t)p.Wb * 4 * N * 4);
     p.total = o;
     return p;
@@ -314,8 +319,8 @@ struct Impl {
       if constexpr (AccumCfg<C>::DFP)
         GZ_CHECK(cudaFuncSetAttribute(k_accum<C, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
-      GZ_CHECK(cudaFuncSetAttribute(k_reduce_win<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    (int)((size_t)threads * 4 * N * 4)));
+      GZ_CHECK(cudaFuncSetAttribute(k_reduce_bits<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)((size_t)RB_THREADS * 4 * N * 4)));
       GZ_CHECK(cudaFuncSetAttribute(k_heavy_tree<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)((size_t)HEAVY_THREADS * 4 * N * 4)));
       attr_set = true;
@@ -380,16 +385,21 @@ struct Impl {
       const int t_lo = p.consolidated ? 0 : gr.t_lo;
       const uint32_t G = p.B / gr.seg;
       const uint32_t total = (uint32_t)gw * G;
+      uint32_t* segT = U(p.o_seg);
+      uint32_t* segR = segT + p.seg_stride;
       k_reduce_seg<C><<<(total + threads - 1) / threads, threads, 0, ss>>>(U(p.o_buckets), U(p.o_offsets), t_lo, gw,
-                                                                           p.B, gr.seg, U(p.o_seg));
+                                                                           p.B, gr.seg, segT, segR);
       GZ_CHECK(cudaGetLastError());
-      const size_t rsmem = (size_t)threads * 4 * N * 4;
-      const uint32_t nb = (G + WIN_PER_BLOCK - 1) / WIN_PER_BLOCK;
-      k_reduce_win<C><<<dim3(nb, gw), threads, rsmem, ss>>>(U(p.o_seg), G, WIN_PER_BLOCK, U(p.o_mid));
+      const int NB = ilog2_u64(G);
+      const uint32_t nsl = (G + RB_PER - 1) / RB_PER;
+      const size_t rsmem = (size_t)RB_THREADS * 4 * N * 4;
+      k_reduce_bits<C><<<dim3(nsl, NB + 1, gw), RB_THREADS, rsmem, ss>>>(segT, segR, G, NB, nsl, U(p.o_mid));
       GZ_CHECK(cudaGetLastError());
-      k_reduce_win<C><<<dim3(1, gw), threads, rsmem, ss>>>(U(p.o_mid), nb, nb, U(p.o_win) + (size_t)t_lo * 4 * N);
+      k_reduce_bits_fin<C><<<dim3(NB + 1, gw), 32, 0, ss>>>(U(p.o_mid), G, NB, nsl, ilog2_u64(gr.seg), U(p.o_terms));
       GZ_CHECK(cudaGetLastError());
-      launches += 3;
+      k_reduce_bits_sum<C><<<gw, 32, 0, ss>>>(U(p.o_terms), NB, U(p.o_win) + (size_t)t_lo * 4 * N);
+      GZ_CHECK(cudaGetLastError());
+      launches += 4;
       ev_reduced = profile_event(prof, ss);
       // a7 (+ a8 on the last group): Horner over the group's windows
       const int last = gi == ngroups - 1;

@@ -575,15 +575,29 @@ __global__ void __launch_bounds__(128) k_heavy_final(const uint32_t* __restrict_
 }
 
 // ------------------------------------------------- a6 bucket reduction
-// Thread (t, g) owns buckets j = g*s+1 .. g*s+s of window t_lo + t (digit j is
-// stored at index j-1).  Running sums from the top give R = sum_u X_u and
-// T = sum_u (u+1) X_u; the segment's share of W_t = sum_j j B_j is
-// T + (g s) R (PAPER.md:239's prefix-sum reduction, segmented).  seg_out is
-// indexed by the group-local id (t - t_lo) * G + g.
+// W_t = sum_{j=1..B} j B_{t,j} (PAPER.md:239's prefix-sum bucket reduction),
+// split so that every stage is either throughput-bound or short:
+//   bucket j = g s + u + 1 (segment g < G = B/s, u < s):
+//   W_t = sum_g T_g + s sum_g g R_g,   T_g = sum_u (u+1) B_{gs+u+1},  R_g = sum_u B_{gs+u+1}
+//       = sum_g T_g + sum_k 2^(k + log2 s) S_k,   S_k = sum_{g : bit k of g} R_g.
+// k_reduce_seg: T_g, R_g by running sums (2s adds per thread, all windows at
+//   once: the only stage with real work, 2 adds per bucket).
+// k_reduce_bits: the plain sums S_k (k < NB = log2 G) and A = sum_g T_g, in
+//   slices of RB_PER elements per CTA (strided serial adds, then a shared-
+//   memory tree).
+// k_reduce_bits_fin: one warp per (set, window): sum of the slice partials
+//   (lane-parallel adds + shuffle tree), then 2^(k + log2 s) by cooperative
+//   doublings.
+// k_reduce_bits_sum: one warp per window: W_t = sum of its NB + 1 terms.
+// The per-segment scalar multiple (g s) R_g of a plain segmented running sum
+// (a 15-bit double-and-add per thread) is gone; its work is now ~NB/2 adds
+// per segment, all in plain sums.
+// Group-local window index t (window t_lo + t); arrays are window-major.
 template <class C>
-__global__ void __launch_bounds__(128) k_reduce_seg(const uint32_t* __restrict__ buckets,
-                                                    const uint32_t* __restrict__ offsets, int t_lo, int W,
-                                                    uint32_t B, int s, uint32_t* __restrict__ seg_out) {
+__global__ void __launch_bounds__(128, 2) k_reduce_seg(const uint32_t* __restrict__ buckets,
+                                                       const uint32_t* __restrict__ offsets, int t_lo, int W,
+                                                       uint32_t B, int s, uint32_t* __restrict__ segT,
+                                                       uint32_t* __restrict__ segR) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
   const uint32_t G = B / s;
@@ -595,42 +609,46 @@ __global__ void __launch_bounds__(128) k_reduce_seg(const uint32_t* __restrict__
     EC_::set_inf(T);
     for (int u = s - 1; u >= 0; --u) {
       const uint32_t key = t * B + g * s + u;
-      if (offsets[key + 1] != offsets[key]) {
+      if (__ldg(offsets + key + 1) != __ldg(offsets + key)) {
         typename EC_::Xyzz X;
         EC_::load(X, buckets + (size_t)key * 4 * N);
         ec_add_hot<C>(R, X);
       }
       ec_add_hot<C>(T, R);
     }
-    ec_mul_small<C>(R, g * (uint32_t)s);      // one out-of-line call per thread
-    ec_add_hot<C>(T, R);
-    EC_::store(seg_out + (size_t)id * 4 * N, T);
+    EC_::store(segT + (size_t)id * 4 * N, T);
+    EC_::store(segR + (size_t)id * 4 * N, R);
   }
 }
 
-// Group sums: group t holds G consecutive XYZZ points; block (b, t) sums the
-// slice [b*per_block, (b+1)*per_block) of group t into out[t*gridDim.x + b].
-// Launched twice (many blocks per window, then one block per window) so the
-// single-window case (weighted points, 2^19 buckets) is not one block's job.
+constexpr uint32_t RB_PER = 512;          // set elements per k_reduce_bits CTA
+constexpr int RB_THREADS = 128;
+
+// set k < NB: the G/2 segments g with bit k set (e-th such g: insert a 1 at
+// bit k of e); set NB: all G segments of segT.  CTA (slice, k, t) writes
+// mid[((t (NB+1) + k) nsl + slice].
 template <class C>
-__global__ void __launch_bounds__(128) k_reduce_win(const uint32_t* __restrict__ seg_out, uint32_t G,
-                                                    uint32_t per_block, uint32_t* __restrict__ win_out) {
+__global__ void __launch_bounds__(RB_THREADS) k_reduce_bits(const uint32_t* __restrict__ segT,
+                                                            const uint32_t* __restrict__ segR, uint32_t G, int NB,
+                                                            uint32_t nsl, uint32_t* __restrict__ mid) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
   extern __shared__ __align__(16) uint32_t red_smem[];
-  const uint32_t t = blockIdx.y;
-  const uint32_t lo = blockIdx.x * per_block;
-  const uint32_t hi = min(G, lo + per_block);
+  const uint32_t slice = blockIdx.x, k = blockIdx.y, t = blockIdx.z;
+  const uint32_t size = (int)k < NB ? G / 2 : G;
+  const uint32_t lo = slice * RB_PER, hi = min(size, lo + RB_PER);
+  const uint32_t* src = ((int)k < NB ? segR : segT) + (size_t)t * G * 4 * N;
   typename EC_::Xyzz acc;
   EC_::set_inf(acc);
-  for (uint32_t g = lo + threadIdx.x; g < hi; g += blockDim.x) {
+  for (uint32_t e = lo + threadIdx.x; e < hi; e += RB_THREADS) {
+    const uint32_t g = (int)k < NB ? (((e >> k) << (k + 1)) | (1u << k) | (e & ((1u << k) - 1u))) : e;
     typename EC_::Xyzz X;
-    EC_::load(X, seg_out + ((size_t)t * G + g) * 4 * N);
+    EC_::load(X, src + (size_t)g * 4 * N);
     ec_add_hot<C>(acc, X);
   }
   EC_::store(red_smem + threadIdx.x * 4 * N, acc);
   __syncthreads();
-  for (uint32_t w = blockDim.x / 2; w > 0; w >>= 1) {
+  for (uint32_t w = RB_THREADS / 2; w > 0; w >>= 1) {
     if (threadIdx.x < w) {
       typename EC_::Xyzz X;
       EC_::load(X, red_smem + (threadIdx.x + w) * 4 * N);
@@ -639,7 +657,70 @@ __global__ void __launch_bounds__(128) k_reduce_win(const uint32_t* __restrict__
     }
     __syncthreads();
   }
-  if (threadIdx.x == 0) EC_::store(win_out + ((size_t)t * gridDim.x + blockIdx.x) * 4 * N, acc);
+  if (threadIdx.x == 0) EC_::store(mid + ((size_t)(t * (NB + 1) + k) * nsl + slice) * 4 * N, acc);
+}
+
+// lane-parallel sum of a warp's points through shared memory (sm: 32 x 4N
+// words): lanes < o add lane o + their index, 5 levels; lane 0 ends with the
+// total.  (Shuffled operands feeding the out-of-line N >= 24 group law
+// miscompile, see CoopEC::level, so the exchange goes through memory.)
+template <class C>
+GZ_DEV void warp_sum(typename EC<C>::Xyzz& acc, uint32_t* sm) {
+  constexpr int N = C::N;
+  const int lane = threadIdx.x & 31;
+  for (int o = 16; o > 0; o >>= 1) {
+    EC<C>::store(sm + lane * 4 * N, acc);
+    __syncwarp();
+    if (lane < o) {
+      typename EC<C>::Xyzz X;
+      EC<C>::load(X, sm + (lane + o) * 4 * N);
+      ec_add_hot<C>(acc, X);
+    }
+    __syncwarp();
+  }
+}
+
+// <<<(NB+1, W), 32>>>: S_k (or A) from its slice partials, times 2^(k + log2 s)
+template <class C>
+__global__ void __launch_bounds__(32) k_reduce_bits_fin(const uint32_t* __restrict__ mid, uint32_t G, int NB,
+                                                        uint32_t nsl, int log_s, uint32_t* __restrict__ terms) {
+  using EC_ = EC<C>;
+  using CO = CoopEC<C>;
+  constexpr int N = C::N;
+  const uint32_t k = blockIdx.x, t = blockIdx.y;
+  const uint32_t size = (int)k < NB ? G / 2 : G;
+  const uint32_t used = (size + RB_PER - 1) / RB_PER;
+  const uint32_t* src = mid + (size_t)(t * (NB + 1) + k) * nsl * 4 * N;
+  typename EC_::Xyzz acc;
+  EC_::set_inf(acc);
+  for (uint32_t q = threadIdx.x; q < used; q += 32) {
+    typename EC_::Xyzz X;
+    EC_::load(X, src + (size_t)q * 4 * N);
+    ec_add_hot<C>(acc, X);
+  }
+  __shared__ __align__(16) uint32_t sm[32 * 4 * N];
+  warp_sum<C>(acc, sm);
+  if (threadIdx.x == 0) EC_::store(sm, acc);
+  __syncwarp();
+  EC_::load(acc, sm);                   // every lane holds the sum (CoopEC)
+  if ((int)k < NB)
+    for (int d = 0; d < (int)k + log_s; ++d) CO::dbl(acc);
+  if (threadIdx.x == 0) EC_::store(terms + (size_t)(t * (NB + 1) + k) * 4 * N, acc);
+}
+
+// <<<W, 32>>>: W_t = sum of the window's NB + 1 terms (NB + 1 <= 32)
+template <class C>
+__global__ void __launch_bounds__(32) k_reduce_bits_sum(const uint32_t* __restrict__ terms, int NB,
+                                                        uint32_t* __restrict__ win_out) {
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  const uint32_t t = blockIdx.x;
+  typename EC_::Xyzz acc;
+  EC_::set_inf(acc);
+  if ((int)threadIdx.x <= NB) EC_::load(acc, terms + (size_t)(t * (NB + 1) + threadIdx.x) * 4 * N);
+  __shared__ __align__(16) uint32_t sm[32 * 4 * N];
+  warp_sum<C>(acc, sm);
+  if (threadIdx.x == 0) EC_::store(win_out + (size_t)t * 4 * N, acc);
 }
 
 // ----------------------------------------- a7 window combination + a8 output
