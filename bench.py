@@ -448,21 +448,24 @@ def main():
     flush_l2 = input_bytes < 2 * L2_BYTES
     flush_buf = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device="cuda") if flush_l2 else None
 
+    # the clock sampler starts first; the warm-up steps then run right before
+    # the timed region, so the timed steps never follow an idle (down-clocked) GPU
+    gz.set_profiling(True)
+    sampler = ClockSampler(local)
+    sampler.start()
+    time.sleep(0.3)
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    gz.set_profiling(True)
     gz.profile_read(reset=True)
-    sampler = ClockSampler(local)
-    sampler.start()
-    time.sleep(0.3)
 
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
+    step_ms = []
     if flush_l2:
         # per-step events, L2 flushed between steps outside the timed windows
         total_ms = 0.0
@@ -474,14 +477,18 @@ def main():
             e1.record(stream)
             torch.cuda.synchronize()
             total_ms += e0.elapsed_time(e1)
+            step_ms.append(round(e0.elapsed_time(e1), 3))
     else:
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for _ in range(args.steps):
+        # one event per step boundary (diagnostic per-step times; the total
+        # is still first-to-last over the K back-to-back steps)
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
+        evs[0].record(stream)
+        for q in range(args.steps):
             step()
-        e1.record(stream)
+            evs[q + 1].record(stream)
         torch.cuda.synchronize()
-        total_ms = e0.elapsed_time(e1)
+        total_ms = evs[0].elapsed_time(evs[-1])
+        step_ms = [round(evs[q].elapsed_time(evs[q + 1]), 3) for q in range(args.steps)]
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -616,7 +623,7 @@ def main():
                        "window_bits": int(prof["c"]), "parallelism": f"shard{world}" if world > 1 else "single",
                        "l2": "flushed between steps" if flush_l2 else f"inputs {input_bytes >> 20} MiB/GPU > L2"},
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "prepared": prepared,
-            "gpu_launches": launches * args.steps,
+            "gpu_launches": launches * args.steps, "step_ms": step_ms,
         }
         print(json.dumps(line), flush=True)
     if comm is not None:

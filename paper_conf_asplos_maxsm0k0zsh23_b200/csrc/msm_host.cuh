@@ -35,7 +35,7 @@ struct Plan {
   uint64_t E_max = 0, chunks_max = 0;
   // workspace byte offsets
   size_t o_pts = 0, o_codes = 0, o_counts = 0, o_offsets = 0, o_cursor = 0, o_tiles = 0, o_vals = 0,
-         o_spay = 0, o_heavy = 0, o_hlist = 0, o_hjobs = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_terms = 0, o_win = 0, total = 0;
+         o_spay = 0, o_heavy = 0, o_hlist = 0, o_hjobs = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_terms = 0, o_hot = 0, o_win = 0, total = 0;
   size_t seg_stride = 0;  // points between segT and segR in o_seg
   struct Grp {
     int t_lo, t_hi;             // windows (inclusive)
@@ -185,6 +185,7 @@ struct Impl {
     p.o_pts = prepared ? 0 : take(n * 2 * N * 4);
     p.o_codes = take((size_t)p.W * n * 4);
     p.o_counts = take((size_t)p.M * 4);
+    p.o_hot = take(((size_t)p.M + 31) / 32 * 4);
     p.o_offsets = take(((size_t)p.M + 1) * 4);
     p.o_cursor = take((size_t)p.M * 4);
     p.o_tiles = take(SCAN_TILE * 4);
@@ -267,6 +268,7 @@ struct Impl {
     }
     // a2: digits + histogram
     GZ_CHECK(cudaMemsetAsync(U(p.o_counts), 0, (size_t)p.M * 4, s));
+    GZ_CHECK(cudaMemsetAsync(U(p.o_hot), 0, ((size_t)p.M + 31) / 32 * 4, s));
     GZ_CHECK(cudaMemsetAsync(U(p.o_heavy), 0, 4 * (p.groups.size() + 4), s));
     const uint32_t bpw = (uint32_t)((n + DIGIT_THREADS - 1) / DIGIT_THREADS);
     const uint32_t key_stride = p.consolidated ? 0u : p.B;
@@ -275,13 +277,13 @@ struct Impl {
     GZ_CHECK(cudaGetLastError());
     // exclusive scan -> offsets (+ cursor copy); offsets[M] = E
     const uint32_t ntiles = (uint32_t)((p.M + SCAN_TILE - 1) / SCAN_TILE);
-    k_scan_tiles<<<ntiles, SCAN_THREADS, 0, s>>>(U(p.o_counts), U(p.o_offsets), p.M, U(p.o_tiles));
+    k_scan_tiles<<<ntiles, SCAN_THREADS, 0, s>>>(U(p.o_counts), U(p.o_offsets), p.M, U(p.o_tiles), U(p.o_hot));
     k_scan_top<<<1, SCAN_THREADS, 0, s>>>(U(p.o_tiles), ntiles, U(p.o_offsets) + p.M);
     k_scan_add<<<ntiles, SCAN_THREADS, 0, s>>>(U(p.o_offsets), U(p.o_cursor), p.M, U(p.o_tiles));
     // a3: scatter into bucket order (window-major grid)
     const uint32_t bpw_s = (uint32_t)((n + SCATTER_TILE - 1) / SCATTER_TILE);
     k_scatter<<<(unsigned)((uint64_t)bpw_s * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw_s, key_stride,
-                                                                         p.val_stride, U(p.o_cursor), U(p.o_vals));
+                                                                         p.val_stride, U(p.o_hot), U(p.o_cursor), U(p.o_vals));
     GZ_CHECK(cudaGetLastError());
     launches += 5;
     cudaEvent_t ev_sorted = profile_event(prof, s);
@@ -312,10 +314,18 @@ struct Impl {
       const char* e = getenv("GZKP_DFP");
       return AccumCfg<C>::DFP && (e ? atoi(e) != 0 : AccumCfg<C>::DFP_DEFAULT);
     }();
+    // GZKP_ACCUM_MINB=3: the BLS12-381 hot loop compiled for 3 CTAs / SM
+    static const bool minb3 = [] {
+      const char* e = getenv("GZKP_ACCUM_MINB");
+      return AccumCfg<C>::DFP && e && atoi(e) == 3;
+    }();
     static bool attr_set = false;
     if (!attr_set) {
       GZ_CHECK(cudaFuncSetAttribute(k_accum<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                     (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
+      if constexpr (AccumCfg<C>::DFP)
+        GZ_CHECK(cudaFuncSetAttribute(k_accum<C, false, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                      (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
       if constexpr (AccumCfg<C>::DFP)
         GZ_CHECK(cudaFuncSetAttribute(k_accum<C, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                       (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
@@ -339,6 +349,9 @@ struct Impl {
         if (mixed)
           k_accum<C, true><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
                                                                    U(p.o_buckets), U(p.o_spay));
+        else if (minb3)
+          k_accum<C, false, 3><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
+                                                                       U(p.o_buckets), U(p.o_spay));
         else
           k_accum<C><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
                                                              U(p.o_buckets), U(p.o_spay));

@@ -118,10 +118,17 @@ GZ_DEV int hot_slot(uint32_t* s_key, uint32_t key) {
 // ----------------------------------------------- a2 digits + histogram
 // One thread per point.  The block stages its scalars in shared memory
 // (coalesced 16-B loads; [word][thread] layout, conflict-free), each thread
-// derives all W digits, writes the digit codes window-major (codes[t*n + i],
-// coalesced) and counts them into the global bucket histogram with
-// warp-aggregated atomics, block-aggregated for hot keys (above).
+// derives all W digits and writes the digit codes window-major (codes[t*n + i],
+// coalesced).  Counting: warp match (match.any) is an MIO instruction with low
+// throughput and ncu r02 showed k_digits / k_scatter MIO-bound, so it is used
+// only where keys repeat: small digits |d| <= DIG_SMALL (the 0 / 1 / small-
+// integer skew of the paper's witness) count into a shared-memory
+// table flushed once per block; other keys go straight to a global RED unless
+// the warp sees a key equal to its lane^1 or lane^2 neighbour's (repeated large
+// digits, e.g. equal scalars), which takes the warp-aggregated path.
 constexpr int DIGIT_THREADS = 256;
+constexpr uint32_t DIG_SMALL = 16;
+constexpr int DIG_SMALL_WIN = 64;             // small table: W <= 64 windows
 template <class C>
 __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __restrict__ sc, size_t n, int c, int W,
                                                           uint32_t key_stride, uint32_t* __restrict__ codes,
@@ -129,10 +136,13 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
   constexpr int NS = C::NS;
   __shared__ uint32_t s_sc[NS * DIGIT_THREADS];
   __shared__ uint32_t s_key[HOT_SLOTS], s_cnt[HOT_SLOTS];
+  __shared__ uint32_t s_small[DIG_SMALL_WIN * DIG_SMALL];
   const size_t base = (size_t)blockIdx.x * DIGIT_THREADS;
   const size_t left = n > base ? n - base : 0;
   const int rows = left < (size_t)DIGIT_THREADS ? (int)left : DIGIT_THREADS;
+  const bool use_small = W <= DIG_SMALL_WIN;
   if (threadIdx.x < HOT_SLOTS) { s_key[threadIdx.x] = HOT_EMPTY; s_cnt[threadIdx.x] = 0; }
+  for (int q = threadIdx.x; q < DIG_SMALL_WIN * (int)DIG_SMALL; q += DIGIT_THREADS) s_small[q] = 0;
   // coalesced staging: the block's scalars are rows*NS contiguous words
   for (int q = threadIdx.x; q < rows * NS; q += DIGIT_THREADS) {
     const int r = q / NS, w = q % NS;
@@ -147,19 +157,37 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
   for (int t = 0; t < W; ++t) {
     const uint32_t code = live ? digit_code(booth_digit(word, t, c)) : 0u;
     if (live) codes[(size_t)t * n + i] = code;
-    if (code) {
-      const uint32_t key = (uint32_t)t * key_stride + (code & ~VAL_NEG) - 1u;
-      const unsigned peers = __match_any_sync(__activemask(), key);
-      if (lane == __ffs(peers) - 1) {
-        const uint32_t cnt = (uint32_t)__popc(peers);
-        const int h = cnt >= HOT_MIN ? hot_slot(s_key, key) : -1;
-        if (h >= 0) atomicAdd(&s_cnt[h], cnt);
-        else atomicAdd(&counts[key], cnt);
+    const uint32_t mag = code & ~VAL_NEG;
+    const uint32_t key = (uint32_t)t * key_stride + mag - 1u;
+    const bool small = code && use_small && mag <= DIG_SMALL;
+    if (__any_sync(0xffffffffu, small) && small) {       // skewed inputs: many lanes share a small digit
+      const unsigned peers = __match_any_sync(__activemask(), mag);
+      if (lane == __ffs(peers) - 1) atomicAdd(&s_small[t * DIG_SMALL + mag - 1], (uint32_t)__popc(peers));
+    }
+    const bool big = code && !small;
+    const uint32_t k_or = big ? key : 0xffffffffu - (uint32_t)lane;    // distinct sentinels
+    const uint32_t nb1 = __shfl_xor_sync(0xffffffffu, k_or, 1);   // every lane shuffles
+    const uint32_t nb2 = __shfl_xor_sync(0xffffffffu, k_or, 2);
+    const bool rep = big && (k_or == nb1 || k_or == nb2);
+    if (__any_sync(0xffffffffu, rep)) {
+      if (big) {
+        const unsigned peers = __match_any_sync(__activemask(), key);
+        if (lane == __ffs(peers) - 1) {
+          const uint32_t cnt = (uint32_t)__popc(peers);
+          const int h = cnt >= HOT_MIN ? hot_slot(s_key, key) : -1;
+          if (h >= 0) atomicAdd(&s_cnt[h], cnt);
+          else atomicAdd(&counts[key], cnt);
+        }
       }
+    } else if (big) {
+      atomicAdd(&counts[key], 1u);
     }
   }
   __syncthreads();
   if (tid < HOT_SLOTS && s_key[tid] != HOT_EMPTY) atomicAdd(&counts[s_key[tid]], s_cnt[tid]);
+  if (use_small)
+    for (int q = tid; q < W * (int)DIG_SMALL; q += DIGIT_THREADS)
+      if (s_small[q]) atomicAdd(&counts[(uint32_t)(q / DIG_SMALL) * key_stride + q % DIG_SMALL], s_small[q]);
 }
 
 // Cross-window consolidation (§4.1; NEXT-1): with prepared
@@ -177,8 +205,14 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
 constexpr int SCATTER_THREADS = 256;
 constexpr int SCATTER_PER_THREAD = 4;        // consecutive points of one window per thread (one 16-B load)
 constexpr int SCATTER_TILE = SCATTER_THREADS * SCATTER_PER_THREAD;
+// A key is "hot" (hotbits, set by k_scan_tiles from the exact histogram) when
+// its bucket holds more than HOT_COUNT entries: only hot keys take the warp
+// match + block reservation path; every other entry reserves its slot with
+// one returning atomic (same-address contention <= HOT_COUNT per key).
+constexpr uint32_t HOT_COUNT = 1024;
 static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32_t* __restrict__ codes, size_t n,
                                                              uint32_t bpw, uint32_t key_stride, uint32_t val_stride,
+                                                             const uint32_t* __restrict__ hotbits,
                                                              uint32_t* __restrict__ cursor, uint32_t* __restrict__ vals) {
   __shared__ uint32_t s_key[HOT_SLOTS], s_cnt[HOT_SLOTS], s_base[HOT_SLOTS];
   const int tid = threadIdx.x;
@@ -199,31 +233,44 @@ static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32
   unsigned peers[SCATTER_PER_THREAD];
   int leader[SCATTER_PER_THREAD], h[SCATTER_PER_THREAD];
   uint32_t pos[SCATTER_PER_THREAD];
+  bool hot[SCATTER_PER_THREAD];
+  bool any_hot = false;
 #pragma unroll
   for (int q = 0; q < SCATTER_PER_THREAD; ++q) {
     peers[q] = 0; leader[q] = 0; h[q] = -1; pos[q] = 0;
     const uint32_t key = t * key_stride + (code[q] & ~VAL_NEG) - 1u;
-    if (!__any_sync(0xffffffffu, code[q] != 0)) continue;        // sparse windows: mostly empty
-    if (code[q]) {
-      peers[q] = __match_any_sync(__activemask(), key);
-      leader[q] = __ffs(peers[q]) - 1;
-      if (lane == leader[q]) {
-        const uint32_t cnt = (uint32_t)__popc(peers[q]);
-        h[q] = cnt >= HOT_MIN ? hot_slot(s_key, key) : -1;
-        if (h[q] >= 0) pos[q] = atomicAdd(&s_cnt[h[q]], cnt);     // offset inside the block's run
-        else pos[q] = atomicAdd(&cursor[key], cnt);
+    hot[q] = code[q] && ((__ldg(hotbits + (key >> 5)) >> (key & 31)) & 1u);
+    if (code[q] && !hot[q]) pos[q] = atomicAdd(&cursor[key], 1u);
+    any_hot |= hot[q];
+  }
+  if (__syncthreads_or(any_hot)) {
+#pragma unroll
+    for (int q = 0; q < SCATTER_PER_THREAD; ++q) {
+      const uint32_t key = t * key_stride + (code[q] & ~VAL_NEG) - 1u;
+      if (!__any_sync(0xffffffffu, hot[q])) continue;
+      if (hot[q]) {
+        peers[q] = __match_any_sync(__activemask(), key);
+        leader[q] = __ffs(peers[q]) - 1;
+        if (lane == leader[q]) {
+          const uint32_t cnt = (uint32_t)__popc(peers[q]);
+          h[q] = cnt >= HOT_MIN ? hot_slot(s_key, key) : -1;
+          if (h[q] >= 0) pos[q] = atomicAdd(&s_cnt[h[q]], cnt);     // offset inside the block's run
+          else pos[q] = atomicAdd(&cursor[key], cnt);
+        }
       }
     }
+    __syncthreads();
+    if (tid < HOT_SLOTS && s_key[tid] != HOT_EMPTY) s_base[tid] = atomicAdd(&cursor[s_key[tid]], s_cnt[tid]);
+    __syncthreads();
   }
-  __syncthreads();
-  if (tid < HOT_SLOTS && s_key[tid] != HOT_EMPTY) s_base[tid] = atomicAdd(&cursor[s_key[tid]], s_cnt[tid]);
-  __syncthreads();
 #pragma unroll
   for (int q = 0; q < SCATTER_PER_THREAD; ++q) {
     if (code[q]) {
       uint32_t p = pos[q];
-      if (lane == leader[q] && h[q] >= 0) p += s_base[h[q]];
-      p = __shfl_sync(peers[q], p, leader[q]) + __popc(peers[q] & ((1u << lane) - 1u));
+      if (hot[q]) {
+        if (lane == leader[q] && h[q] >= 0) p += s_base[h[q]];
+        p = __shfl_sync(peers[q], p, leader[q]) + __popc(peers[q] & ((1u << lane) - 1u));
+      }
       vals[p] = (t * val_stride + (uint32_t)(i0 + q)) | (code[q] & VAL_NEG);
     }
   }
@@ -260,7 +307,7 @@ GZ_DEV uint32_t block_exclusive_scan(uint32_t v, uint32_t* warp_sums, uint32_t* 
 }
 
 static __global__ void k_scan_tiles(const uint32_t* __restrict__ in, uint32_t* __restrict__ out, uint32_t M,
-                             uint32_t* __restrict__ tile_sums) {
+                             uint32_t* __restrict__ tile_sums, uint32_t* __restrict__ hotbits) {
   __shared__ uint32_t ws[32];
   const size_t base = (size_t)blockIdx.x * SCAN_TILE + threadIdx.x * SCAN_PER_THREAD;
   uint32_t v[SCAN_PER_THREAD], s = 0;
@@ -268,6 +315,7 @@ static __global__ void k_scan_tiles(const uint32_t* __restrict__ in, uint32_t* _
   for (int k = 0; k < SCAN_PER_THREAD; ++k) {
     v[k] = (base + k < M) ? in[base + k] : 0u;
     s += v[k];
+    if (v[k] > HOT_COUNT) atomicOr(&hotbits[(base + k) >> 5], 1u << ((base + k) & 31));   // hotbits zeroed by the host
   }
   uint32_t total;
   uint32_t ex = block_exclusive_scan(s, ws, &total);
@@ -378,8 +426,10 @@ struct AccumCfg {
 // (threads past the group's real chunk count exit): while the next group
 // accumulates, finishing CTAs free slots for the high-priority side stream
 // that merges / reduces / combines the previous group.
-template <class C, bool MIXED = false>
-__global__ void __launch_bounds__(128, AccumCfg<C>::MIN_CTAS)
+// MINB overrides the register budget (GZKP_ACCUM_MINB=3 selects 3 CTAs / SM,
+// <= 168 registers, for BLS12-381; see msm_host.cuh).
+template <class C, bool MIXED = false, int MINB = AccumCfg<C>::MIN_CTAS>
+__global__ void __launch_bounds__(128, MINB)
     k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off, Group grp,
             const uint32_t* __restrict__ pts, int S, uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay) {
   using Fp = Field<C>;
