@@ -45,6 +45,8 @@ WORKLOADS = {
     "bls12_381_2p26_sparse": ("bls12_381", 26, 5, "zcash_like", "BLS12-381 G1 MSM n=2^26, sparse/skewed scalars"),
     "bls12_381_2p26": ("bls12_381", 26, 6, "uniform", "BLS12-381 G1 MSM n=2^26, uniform scalars"),
     "bn254_2p10": ("bn254", 10, 1, "uniform", "BN254 G1 MSM n=2^10, uniform random scalars"),
+    # one rank's shard of configs[2] at 8 GPUs (diagnostic: the per-GPU step of the 8-GPU run)
+    "bls12_381_2p19": ("bls12_381", 19, 3, "uniform", "BLS12-381 G1 MSM n=2^19 (one rank's shard of n=2^22 at 8 GPUs)"),
     # G2 (not a BASELINE config: the same MSM over F_p^2)
     "bn254_g2_2p20": ("bn254_g2", 20, 7, "uniform", "BN254 G2 MSM n=2^20, uniform scalars (NEXT-3)"),
     "bls12_381_g2_2p20": ("bls12_381_g2", 20, 8, "uniform", "BLS12-381 G2 MSM n=2^20, uniform scalars (NEXT-3)"),
