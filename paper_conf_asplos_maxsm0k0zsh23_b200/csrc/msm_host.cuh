@@ -35,7 +35,7 @@ struct Plan {
   uint64_t E_max = 0, chunks_max = 0;
   // workspace byte offsets
   size_t o_pts = 0, o_codes = 0, o_counts = 0, o_offsets = 0, o_cursor = 0, o_tiles = 0, o_vals = 0,
-         o_spay = 0, o_heavy = 0, o_hlist = 0, o_hjobs = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_terms = 0, o_hot = 0, o_win = 0, total = 0;
+         o_spay = 0, o_heavy = 0, o_hlist = 0, o_hjobs = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_terms = 0, o_hot = 0, o_cb = 0, o_mcnt = 0, o_win = 0, total = 0;
   size_t seg_stride = 0;  // points between segT and segR in o_seg
   struct Grp {
     int t_lo, t_hi;             // windows (inclusive)
@@ -72,12 +72,27 @@ struct Impl {
       const int W = (C::SCALAR_BITS + 1 + c - 1) / c;
       const double B = std::ldexp(1.0, c - 1);
       const double entries = (double)n * W * (1.0 - std::ldexp(1.0, -c));
-      const double reduce = W * B * 3.4 * add + 60.0 * add * lat / 8.0;
+      // bucket reduction: 2 adds per bucket (k_reduce_seg) + the bit-set sums'
+      // latency (round-1 measurement: 1.17 ms for 16 x 2^15 buckets)
+      const double reduce = W * B * 2.0 * add + 30.0 * add * lat / 8.0;
       const double tail = (W - 1) * (c * dbl + add) * lat;
-      const double cost = entries * madd + reduce + tail;
+      const double cost = entries * madd + reduce + tail + top_window_merge(n, c, W) * add * lat;
       if (cost < best_cost) { best_cost = cost; best = c; }
     }
     return best;
+  }
+
+  // Serial adds the merge of the top window costs: it holds only the
+  // b + 1 - c (W - 1) leftover scalar bits, so its few buckets are heavy
+  // (2^19 points at c = 14: 8 buckets of 2^16 entries, a 2-level heavy tree,
+  // 0.4 ms measured) -- the k_heavy_tree depth, 15 serial adds per level.
+  static double top_window_merge(size_t n, int c, int W) {
+    const int top_bits = C::SCALAR_BITS + 1 - c * (W - 1);
+    const double per_bucket = (double)n / std::ldexp(1.0, std::max(top_bits - 1, 0));
+    const double q = per_bucket / 64.0;               // partials of one top bucket (S = 64)
+    if (q <= 1.0) return 0.0;
+    if (q <= MERGE_QMAX) return q - 1.0;
+    return 15.0 * std::ceil(std::log(q) / std::log((double)HEAVY_SPAN));
   }
 
   // Window size when all windows share one bucket set (weighted points): no
@@ -102,6 +117,38 @@ struct Impl {
     return best;
   }
 
+  // Accumulation chunk size S (entries per thread).  64 by default; for small
+  // shards the grid is a few waves of the resident threads and a partly
+  // filled last wave idles SMs (n = 2^19 at c = 16: 3.46 waves, ~13 % lost),
+  // so S in [40, 64] is picked to make the wave count just below an integer
+  // (E estimated as n W, exact for uniform scalars up to zero digits).
+  static uint64_t accum_resident_threads() {
+    static const uint64_t v = [] {
+      int per_sm = 0;
+      const size_t smem = (size_t)128 * Stage<C>::SLOT_WORDS * 4;
+      if (smem > 48 * 1024 ||
+          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_accum<C>, 128, smem) != cudaSuccess)
+        per_sm = 0;
+      cudaGetLastError();
+      return (uint64_t)per_sm * device_sm_count() * 128;
+    }();
+    return v;
+  }
+  static int chunk_entries_for(uint64_t E) {
+    const uint64_t T = accum_resident_threads();
+    if (!T || E == 0) return 64;
+    auto eff = [&](int S) {
+      const double w = (double)E / ((double)S * (double)T);
+      return w / std::ceil(w);
+    };
+    if ((double)E / (64.0 * (double)T) >= 24.0) return 64;     // many waves: quantisation < 4 %
+    int best = 64;
+    double be = eff(64);
+    for (int S = 63; S >= 40; --S)
+      if (eff(S) > be + 0.02) { be = eff(S); best = S; }
+    return best;
+  }
+
   static Plan plan(size_t n, bool prepared, bool consolidated = false, int c_forced = 0, size_t table_n = 0) {
     Plan p;
     p.n = n;
@@ -116,7 +163,7 @@ struct Impl {
     if (S <= 0) {
       if (const char* e = getenv("GZKP_SEGMENT")) S = atoi(e);
     }
-    if (S <= 0) S = 64;
+    if (S <= 0) S = chunk_entries_for((uint64_t)n * p.W);
     p.S = S;
     // reduction segment: up to 16 buckets, fewer when that leaves < ~32K threads
     {
@@ -191,6 +238,8 @@ struct Impl {
     p.o_tiles = take(SCAN_TILE * 4);
     p.o_vals = take(std::max<uint64_t>(p.E_max, 1) * 4);
     p.o_spay = take(2 * p.chunks_max * 4 * N * 4);
+    p.o_cb = take(p.chunks_max * 8);                       // merge list (uint2 per spanning bucket)
+    p.o_mcnt = take(4 * (p.groups.size() + 1));
     p.o_heavy = take(4 * (p.groups.size() + 4));
     p.o_hlist = take(16 * std::max<uint64_t>(hlist_elems, 1));
     p.o_hjobs = take(4 * (size_t)std::max(p.heavy_levels, 1) * (hlist_elems + p.groups.size()));
@@ -269,6 +318,7 @@ struct Impl {
     // a2: digits + histogram
     GZ_CHECK(cudaMemsetAsync(U(p.o_counts), 0, (size_t)p.M * 4, s));
     GZ_CHECK(cudaMemsetAsync(U(p.o_hot), 0, ((size_t)p.M + 31) / 32 * 4, s));
+    GZ_CHECK(cudaMemsetAsync(U(p.o_mcnt), 0, 4 * (p.groups.size() + 1), s));
     GZ_CHECK(cudaMemsetAsync(U(p.o_heavy), 0, 4 * (p.groups.size() + 4), s));
     const uint32_t bpw = (uint32_t)((n + DIGIT_THREADS - 1) / DIGIT_THREADS);
     const uint32_t key_stride = p.consolidated ? 0u : p.B;
@@ -342,22 +392,24 @@ struct Impl {
     for (int gi = 0; gi < ngroups; ++gi) {
       const auto& gr = p.groups[gi];
       const Group grp{gr.key_lo, gr.key_hi, (uint32_t)gr.chunk_base};
+      uint2* mlist = (uint2*)U(p.o_cb) + gr.chunk_base;
+      uint32_t* mcnt = U(p.o_mcnt) + gi;
       // a4 (main stream)
       cudaEvent_t a0 = profile_event(prof, s);
       const unsigned acc_grid = (unsigned)((gr.chunks_max + acc_threads - 1) / acc_threads);
       if constexpr (AccumCfg<C>::DFP) {
         if (mixed)
           k_accum<C, true><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
-                                                                   U(p.o_buckets), U(p.o_spay));
+                                                                   U(p.o_buckets), U(p.o_spay), mlist, mcnt);
         else if (minb3)
           k_accum<C, false, 3><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
-                                                                       U(p.o_buckets), U(p.o_spay));
+                                                                       U(p.o_buckets), U(p.o_spay), mlist, mcnt);
         else
           k_accum<C><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
-                                                             U(p.o_buckets), U(p.o_spay));
+                                                             U(p.o_buckets), U(p.o_spay), mlist, mcnt);
       } else {
         k_accum<C><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
-                                                           U(p.o_buckets), U(p.o_spay));
+                                                           U(p.o_buckets), U(p.o_spay), mlist, mcnt);
       }
       GZ_CHECK(cudaGetLastError());
       cudaEvent_t a1 = profile_event(prof, s);
@@ -370,12 +422,11 @@ struct Impl {
       }
       // a5 (side stream): boundary partials -> buckets, heavy-bucket tree
       uint32_t* heavy = U(p.o_heavy) + gi;
-      const uint32_t nkeys = gr.key_hi - gr.key_lo;
-      const int gm = (int)std::min<uint64_t>((nkeys + threads - 1) / threads, (uint64_t)sms * 16);
       uint4* hlist = (uint4*)U(p.o_hlist) + gr.hbase;
       uint32_t* hjobs = U(p.o_hjobs) + (size_t)std::max(p.heavy_levels, 1) * (gr.hbase + gi);
-      k_merge_bucket<C><<<gm, threads, 0, ss>>>(U(p.o_offsets), grp, p.S, U(p.o_spay), U(p.o_buckets), heavy, hlist,
-                                                gr.hmax);
+      const int gm = (int)std::min<uint64_t>((gr.chunks_max + threads - 1) / threads, (uint64_t)sms * 16);
+      k_merge_bucket<C><<<gm, threads, 0, ss>>>(U(p.o_offsets), grp, p.S, mlist, mcnt, U(p.o_spay), U(p.o_buckets),
+                                                heavy, hlist, gr.hmax);
       GZ_CHECK(cudaGetLastError());
       if (gr.heavy_levels > 0) {
         k_heavy_plan<<<1, 32, 0, ss>>>(heavy, hlist, gr.hmax, gr.heavy_levels, hjobs);

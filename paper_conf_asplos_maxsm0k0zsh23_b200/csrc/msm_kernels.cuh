@@ -431,7 +431,8 @@ struct AccumCfg {
 template <class C, bool MIXED = false, int MINB = AccumCfg<C>::MIN_CTAS>
 __global__ void __launch_bounds__(128, MINB)
     k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off, Group grp,
-            const uint32_t* __restrict__ pts, int S, uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay) {
+            const uint32_t* __restrict__ pts, int S, uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay,
+            uint2* __restrict__ mlist, uint32_t* __restrict__ mcnt) {
   using Fp = Field<C>;
   using EC_ = EC<C>;
   using St = Stage<C>;
@@ -494,28 +495,42 @@ __global__ void __launch_bounds__(128, MINB)
   }
   cp_async_wait<0>();
   flush(true);
+  // merge list: the chunk in which a spanning bucket STARTS owns its merge
+  // (its last run is open to the right); one warp-aggregated append per warp
+  const bool owner = nxt > end && __ldg(off + cur) >= beg;
+  const unsigned act = __activemask();
+  const unsigned om = __ballot_sync(act, owner);
+  if (om) {
+    const int lane = threadIdx.x & 31, lead = __ffs(om) - 1;
+    uint32_t base = 0;
+    if (lane == lead) base = atomicAdd(mcnt, (uint32_t)__popc(om));
+    base = __shfl_sync(act, base, lead);
+    if (owner) mlist[base + __popc(om & ((1u << lane) - 1u))] = make_uint2(cur, chunk);
+  }
 }
 
 // ----------------------------------------------------------- a5 merge
-// Thread per bucket of the group: a bucket spanning local chunks t0 < t1 has
+// Thread per entry (k, t0) of the merge list that k_accum appended: bucket k
+// starts in local chunk t0 and continues past it, up to chunk t1, so it has
 // q = t1 - t0 + 1 partials (slot 2*(base+t0)+1, then head slots 2*(base+t)).
 // q <= MERGE_QMAX: summed here.  Larger q (a heavy bucket of a skewed input)
 // is appended to the group's heavy list (k, t0, t1) and reduced by the
-// k_heavy_* kernels instead.
+// k_heavy_* kernels instead.  The compact list keeps every lane busy whatever
+// the share of spanning buckets among the keys (small shards: few).
 template <class C>
 __global__ void __launch_bounds__(128) k_merge_bucket(const uint32_t* __restrict__ off, Group grp, int S,
+                                                      const uint2* __restrict__ mlist, const uint32_t* __restrict__ mcnt,
                                                       const uint32_t* __restrict__ spay, uint32_t* __restrict__ buckets,
                                                       uint32_t* __restrict__ heavy_cnt, uint4* __restrict__ hlist,
                                                       uint32_t hmax) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
   const uint32_t G0 = __ldg(off + grp.key_lo);
-  for (uint32_t k = grp.key_lo + blockIdx.x * blockDim.x + threadIdx.x; k < grp.key_hi;
-       k += gridDim.x * blockDim.x) {
-    const uint32_t b0 = __ldg(off + k), b1 = __ldg(off + k + 1);
-    if (b1 == b0) continue;
-    const uint32_t t0 = (b0 - G0) / S, t1 = (b1 - 1 - G0) / S;
-    if (t0 == t1) continue;                              // written by k_accum
+  const uint32_t cnt = *mcnt;
+  for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < cnt; e += gridDim.x * blockDim.x) {
+    const uint2 m = mlist[e];
+    const uint32_t k = m.x, t0 = m.y;
+    const uint32_t t1 = (__ldg(off + k + 1) - 1 - G0) / S;
     if (t1 - t0 + 1 > (uint32_t)MERGE_QMAX) {
       const uint32_t h = atomicAdd(heavy_cnt, 1u);
       if (h < hmax) hlist[h] = make_uint4(k, t0, t1, 0u);   // hmax bounds every input (planner)

@@ -4,8 +4,8 @@ cd "${GRAFT_REPO_ROOT:-/root/repo}"
 mkdir -p gpurun_out
 timeout 420 python -m pytest tests -m gpu -x -q --timeout 120 -p no:cacheprovider > gpurun_out/pytest_gpu.txt 2>&1
 echo "pytest exit $?" >> gpurun_out/pytest_gpu.txt
-for a in "--workload bls12_381_2p22" "--workload bls12_381_2p22 --chunk 128" "--workload bls12_381_2p22 --chunk 256" "--workload bls12_381_2p26_sparse" "--workload bn254_2p20" $EXTRA; do
-  echo "== $a" >> gpurun_out/quick.txt
-  timeout 150 python bench.py $a --steps 5 --no-cpu-baseline --no-e2e --no-prepared 2>>gpurun_out/quick.err \
+for w in ${WORKLOADS:-bls12_381_2p22 bls12_381_2p19 bls12_381_2p26_sparse bn254_2p20 mnt4_753_2p20}; do
+  echo "== $w" >> gpurun_out/quick.txt
+  timeout 150 python bench.py --workload $w --steps 5 --no-cpu-baseline --no-e2e --no-prepared 2>>gpurun_out/quick.err \
     | python -c "import json,sys; d=json.loads(sys.stdin.read()); print(round(d['ms_per_step'],3), d['step_ms'], d['roofline']['phase_ms_per_step'])" >> gpurun_out/quick.txt
 done
