@@ -186,6 +186,12 @@ struct Impl {
       p.groups.push_back({0, p.W - 1, 0, p.M, 0, 0, 0, 0, 0});
     } else if (consolidated) {
       p.groups.push_back({0, p.W - 1, 0, p.B, 0, 0, 0, 0, 0});
+    } else if (pipeline == 2 && p.W >= 2) {
+      // two equal groups: the top half's merge / reduction / Horner run on the
+      // side stream while the bottom half accumulates
+      const int mid = p.W / 2;
+      p.groups.push_back({mid, p.W - 1, (uint32_t)mid * p.B, (uint32_t)p.W * p.B, 0, 0, 0, 0, 0});
+      p.groups.push_back({0, mid - 1, 0, (uint32_t)mid * p.B, 0, 0, 0, 0, 0});
     } else {
       int hi = p.W - 1;
       while (hi >= 0) {
@@ -457,7 +463,8 @@ struct Impl {
       const int NB = ilog2_u64(G);
       const uint32_t nsl = (G + RB_PER - 1) / RB_PER;
       const size_t rsmem = (size_t)RB_THREADS * 4 * N * 4;
-      k_reduce_bits<C><<<dim3(nsl, NB + 1, gw), RB_THREADS, rsmem, ss>>>(segT, segR, G, NB, nsl, U(p.o_mid));
+      const uint32_t nslR = (G / 2 + RB_PER - 1) / RB_PER;
+      k_reduce_bits<C><<<dim3(NB * nslR + nsl, gw), RB_THREADS, rsmem, ss>>>(segT, segR, G, NB, nsl, U(p.o_mid));
       GZ_CHECK(cudaGetLastError());
       k_reduce_bits_fin<C><<<dim3(NB + 1, gw), 32, 0, ss>>>(U(p.o_mid), G, NB, nsl, ilog2_u64(gr.seg), U(p.o_terms));
       GZ_CHECK(cudaGetLastError());

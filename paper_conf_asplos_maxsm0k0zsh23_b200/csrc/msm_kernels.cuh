@@ -690,16 +690,22 @@ constexpr uint32_t RB_PER = 512;          // set elements per k_reduce_bits CTA
 constexpr int RB_THREADS = 128;
 
 // set k < NB: the G/2 segments g with bit k set (e-th such g: insert a 1 at
-// bit k of e); set NB: all G segments of segT.  CTA (slice, k, t) writes
-// mid[((t (NB+1) + k) nsl + slice].
+// bit k of e); set NB: all G segments of segT.  The grid is exact, (slices of
+// all sets, W): blockIdx.x < NB nslR are the R-set slices (set x / nslR),
+// the rest the T-set's; CTA (k, slice) writes mid[((t (NB+1) + k) nsl + slice]
+// (nsl = the T-set's slice count).  3 CTAs / SM so one wave holds the grid.
 template <class C>
-__global__ void __launch_bounds__(RB_THREADS) k_reduce_bits(const uint32_t* __restrict__ segT,
-                                                            const uint32_t* __restrict__ segR, uint32_t G, int NB,
-                                                            uint32_t nsl, uint32_t* __restrict__ mid) {
+__global__ void __launch_bounds__(RB_THREADS, 3) k_reduce_bits(const uint32_t* __restrict__ segT,
+                                                               const uint32_t* __restrict__ segR, uint32_t G, int NB,
+                                                               uint32_t nsl, uint32_t* __restrict__ mid) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
   extern __shared__ __align__(16) uint32_t red_smem[];
-  const uint32_t slice = blockIdx.x, k = blockIdx.y, t = blockIdx.z;
+  const uint32_t nslR = (G / 2 + RB_PER - 1) / RB_PER;
+  const uint32_t x = blockIdx.x, t = blockIdx.y;
+  const bool rset = x < (uint32_t)NB * nslR;
+  const uint32_t k = rset ? x / nslR : (uint32_t)NB;
+  const uint32_t slice = rset ? x % nslR : x - (uint32_t)NB * nslR;
   const uint32_t size = (int)k < NB ? G / 2 : G;
   const uint32_t lo = slice * RB_PER, hi = min(size, lo + RB_PER);
   const uint32_t* src = ((int)k < NB ? segR : segT) + (size_t)t * G * 4 * N;
@@ -730,10 +736,12 @@ __global__ void __launch_bounds__(RB_THREADS) k_reduce_bits(const uint32_t* __re
 // total.  (Shuffled operands feeding the out-of-line N >= 24 group law
 // miscompile, see CoopEC::level, so the exchange goes through memory.)
 template <class C>
-GZ_DEV void warp_sum(typename EC<C>::Xyzz& acc, uint32_t* sm) {
+GZ_DEV void warp_sum(typename EC<C>::Xyzz& acc, uint32_t* sm, int used = 32) {
   constexpr int N = C::N;
   const int lane = threadIdx.x & 31;
-  for (int o = 16; o > 0; o >>= 1) {
+  int top = 1;                                   // levels only over the lanes that hold values
+  while (top < used && top < 32) top <<= 1;
+  for (int o = top >> 1; o > 0; o >>= 1) {
     EC<C>::store(sm + lane * 4 * N, acc);
     __syncwarp();
     if (lane < o) {
@@ -764,7 +772,7 @@ __global__ void __launch_bounds__(32) k_reduce_bits_fin(const uint32_t* __restri
     ec_add_hot<C>(acc, X);
   }
   __shared__ __align__(16) uint32_t sm[32 * 4 * N];
-  warp_sum<C>(acc, sm);
+  warp_sum<C>(acc, sm, (int)min(used, 32u));
   if (threadIdx.x == 0) EC_::store(sm, acc);
   __syncwarp();
   EC_::load(acc, sm);                   // every lane holds the sum (CoopEC)
@@ -784,7 +792,7 @@ __global__ void __launch_bounds__(32) k_reduce_bits_sum(const uint32_t* __restri
   EC_::set_inf(acc);
   if ((int)threadIdx.x <= NB) EC_::load(acc, terms + (size_t)(t * (NB + 1) + threadIdx.x) * 4 * N);
   __shared__ __align__(16) uint32_t sm[32 * 4 * N];
-  warp_sum<C>(acc, sm);
+  warp_sum<C>(acc, sm, NB + 1);
   if (threadIdx.x == 0) EC_::store(win_out + (size_t)t * 4 * N, acc);
 }
 

@@ -2,7 +2,8 @@
 because the switches are read once per process:
 
 * GZKP_DFP=1           hot loop with FP64 (DFP) products (NEXT-2 experiment)
-* GZKP_PIPELINE=1      window-group pipeline on a side stream
+* GZKP_PIPELINE=1      window-group pipeline on a side stream (halving groups)
+* GZKP_PIPELINE=2      two equal window groups
 * GZKP_ACCUM_THREADS=32  small accumulation CTAs
 * GZKP_WINDOW_BITS / GZKP_SEGMENT  planner overrides
 """
@@ -39,7 +40,7 @@ print("VARIANT_OK" if ok else "VARIANT_FAIL")
 """ % ROOT
 
 
-@pytest.mark.parametrize("env", [{"GZKP_DFP": "1"}, {"GZKP_PIPELINE": "1"}, {"GZKP_ACCUM_THREADS": "32"},
+@pytest.mark.parametrize("env", [{"GZKP_DFP": "1"}, {"GZKP_PIPELINE": "1"}, {"GZKP_PIPELINE": "2"}, {"GZKP_ACCUM_THREADS": "32"},
                                  {"GZKP_WINDOW_BITS": "11", "GZKP_SEGMENT": "5"},
                                  {"GZKP_DFP": "1", "GZKP_PIPELINE": "1", "GZKP_ACCUM_THREADS": "64"}],
                          ids=lambda e: ",".join(f"{k}={v}" for k, v in e.items()))
