@@ -17,6 +17,10 @@
 #include "field2.cuh"
 #include "field_dfp.cuh"
 
+#ifndef GZKP_COOP_KARATSUBA
+#define GZKP_COOP_KARATSUBA 0   // 1: Karatsuba products in the cooperative chains (measured slower: BLS12-381 tail 1.01 -> 1.20 ms)
+#endif
+
 namespace gzkp {
 
 template <class C>
@@ -269,8 +273,15 @@ struct CoopEC {
     pick(x, q, x0, x1, x2, x3);
     pick(y, q, y0, y1, y2, y3);
     // always inlined here (also for N = 24): per-lane operands feeding an
-    // out-of-line call between warp shuffles produced wrong MNT4-753 results
+    // out-of-line call between warp shuffles produced wrong MNT4-753 results.
+    // GZKP_COOP_KARATSUBA=1 tries the one-level Karatsuba product here (three
+    // independent half products for the single warp's ILP): measured slower.
+#if GZKP_COOP_KARATSUBA
+    if constexpr (N >= 8 && N <= 12 && N % 4 == 0) Fp::mul_kara(r, x, y);
+    else Fp::mul_inline(r, x, y);
+#else
     Fp::mul_inline(r, x, y);
+#endif
   }
 
   // P = 2P (all lanes hold P; identical result on every lane)
