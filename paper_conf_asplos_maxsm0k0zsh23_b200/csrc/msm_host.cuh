@@ -457,7 +457,14 @@ struct Impl {
       const uint32_t total = (uint32_t)gw * G;
       uint32_t* segT = U(p.o_seg);
       uint32_t* segR = segT + p.seg_stride;
-      k_reduce_seg<C><<<(total + threads - 1) / threads, threads, 0, ss>>>(U(p.o_buckets), U(p.o_offsets), t_lo, gw,
+      // small CTAs spread the ~W 2^(c-1) / s segment threads evenly over the
+      // SMs (32K threads on 148 SMs: 128-thread CTAs leave some SMs at 1 CTA)
+      static const int rcta = [] {
+        const char* e = getenv("GZKP_REDUCE_CTA");
+        const int v = e ? atoi(e) : 64;              // measured: 64 / 32 / 128 = 1.02 / 1.03 / 1.05 ms
+        return (v >= 32 && v <= 128 && v % 32 == 0) ? v : 64;
+      }();
+      k_reduce_seg<C><<<(total + rcta - 1) / rcta, rcta, 0, ss>>>(U(p.o_buckets), U(p.o_offsets), t_lo, gw,
                                                                            p.B, gr.seg, segT, segR);
       GZ_CHECK(cudaGetLastError());
       const int NB = ilog2_u64(G);
