@@ -398,40 +398,11 @@ __device__ __noinline__ void ec_to_affine(uint32_t* x, uint32_t* y, const typena
 // Inlined group law for the throughput-bound post-processing kernels (merge,
 // bucket reduction) when N <= 12: passing XYZZ operands by reference to an
 // out-of-line function keeps them in local memory (r01: k_reduce_seg had a
-// 792-B frame and ran at ~28 % of IMAD peak).  MNT4-753 keeps the calls.
+// 792-B frame and ran at ~28 % of IMAD peak).  N > 12 (MNT4-753 and the G2
+// curves) keeps the calls.
 template <class C>
 GZ_DEV void ec_add_hot(typename EC<C>::Xyzz& A, const typename EC<C>::Xyzz& B) {
   if constexpr (C::N <= 12) EC<C>::add(A, B);
   else ec_add<C>(A, B);
 }
-template <class C>
-GZ_DEV void ec_dbl_hot(typename EC<C>::Xyzz& A) {
-  if constexpr (C::N <= 12) EC<C>::dbl(A);
-  else ec_dbl<C>(A);
-}
-template <class C>
-GZ_DEV void ec_mul_small_hot(typename EC<C>::Xyzz& P, uint32_t k) {
-  using E = EC<C>;
-  if (k == 0 || E::is_inf(P)) { E::set_inf(P); return; }
-  typename E::Xyzz B = P;
-  const int top = 31 - __clz(k);
-  for (int i = top - 1; i >= 0; --i) {
-    ec_dbl_hot<C>(P);
-    if ((k >> i) & 1) ec_add_hot<C>(P, B);
-  }
-}
-
-// P = k * P for a small non-negative integer k (double-and-add, MSB first)
-template <class C>
-__device__ __noinline__ void ec_mul_small(typename EC<C>::Xyzz& P, uint32_t k) {
-  using E = EC<C>;
-  if (k == 0 || E::is_inf(P)) { E::set_inf(P); return; }
-  typename E::Xyzz B = P;
-  const int top = 31 - __clz(k);
-  for (int i = top - 1; i >= 0; --i) {
-    ec_dbl<C>(P);
-    if ((k >> i) & 1) ec_add<C>(P, B);
-  }
-}
-
 }  // namespace gzkp
