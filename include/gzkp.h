@@ -112,9 +112,11 @@ gzkp_status gzkp_msm_host(int curve, const void *points_affine_host, const void 
  *   interval M = 1): the library stores the weighted points 2^(c t) P_i for
  *   every window t (W = ceil((b+1)/c) copies, W*n*2*field_bytes bytes of HBM),
  *   so all windows accumulate into ONE bucket set and the window reduction
- *   disappears.  window_bits = 0 lets the planner choose c; later MSMs on the
- *   handle use that c.
- * weighted = 0: Montgomery-form copy of the points only (standard pipeline).
+ *   disappears.  window_bits = 0 lets the planner choose c, else 2..22; later
+ *   MSMs on the handle use that c.
+ * weighted = 0: Montgomery-form copy of the points only (standard pipeline);
+ *   window_bits 0 (planner per call) or 2..16 (fixed c for every call).
+ *   Other values: GZKP_ERROR_INVALID_VALUE.
  * gzkp_points_prepare = _ex(window_bits 0, weighted 1), falling back to
  * weighted 0 if the table does not fit. */
 gzkp_status gzkp_points_prepare_ex(int curve, const void *points_affine, size_t n, int window_bits,
@@ -208,6 +210,12 @@ int gzkp_window_bits(int curve, size_t n);
  * stats[3] = window bits c of the last call. */
 gzkp_status gzkp_set_profiling(int on);
 gzkp_status gzkp_profile_read(double phase_ms[5], uint64_t stats[4], int reset);
+/* The library keeps one grow-only workspace and one high-priority side stream
+ * per (device, caller stream) so back-to-back calls do not re-allocate.  Call
+ * this before destroying a stream that was passed to the library: it frees
+ * that stream's workspace (stream-ordered, after the work queued on it) and
+ * synchronises and destroys its side stream.  Safe on streams never used. */
+gzkp_status gzkp_release_stream(gzkp_stream stream);
 const char *gzkp_status_string(gzkp_status status);
 const char *gzkp_last_error(void);
 

@@ -78,6 +78,7 @@ def lib():
             "gzkp_ntt": ([i32, vp, vp, i32, i32, vp], i32),
             "gzkp_ntt_last_launches": ([], i32),
             "gzkp_scalar_field_op": ([i32, i32, vp, vp, vp, sz, vp], i32),
+            "gzkp_release_stream": ([vp], i32),
             "gzkp_status_string": ([i32], ctypes.c_char_p),
             "gzkp_last_error": ([], ctypes.c_char_p),
         }
@@ -140,10 +141,29 @@ def _torch():
     return torch
 
 
-def _stream_ptr(stream=None) -> int:
+def _stream_ptr(stream=None, device=None) -> int:
+    """The raw cudaStream_t: `stream` if given, else the current stream of
+    `device` (the device of the call's tensors), else of the current device."""
     torch = _torch()
-    s = stream if stream is not None else torch.cuda.current_stream()
+    s = stream if stream is not None else torch.cuda.current_stream(device)
     return s.cuda_stream
+
+
+def _on(t):
+    """Context manager: make the tensor's GPU the current device for the call
+    (the library launches on the current device)."""
+    return _torch().cuda.device(t.device)
+
+
+def _host_u32(a, cols: int, name: str) -> np.ndarray:
+    """Contiguous [n, cols] u32 host array; the column count must match the
+    curve (the C call copies n*cols*4 bytes from the pointer)."""
+    a = np.ascontiguousarray(a, dtype=np.uint32)
+    if a.ndim == 1 and a.size % cols == 0:
+        a = a.reshape(-1, cols)
+    if a.ndim != 2 or a.shape[1] != cols:
+        raise GzkpError(f"{name}: expected shape [n, {cols}], got {a.shape}")
+    return a
 
 
 def _dev_u32(x, cols: int, name: str):
@@ -157,6 +177,8 @@ def _dev_u32(x, cols: int, name: str):
         x = x.view(torch.int32)
     if x.dtype not in (torch.int32, torch.uint32):
         raise GzkpError(f"{name}: expected int32/uint32/uint8 limbs, got {x.dtype}")
+    if x.numel() % cols or (x.dim() == 2 and x.shape[1] != cols):
+        raise GzkpError(f"{name}: expected [n, {cols}] u32 limbs, got shape {tuple(x.shape)}")
     x = x.contiguous().reshape(-1, cols)
     if x.data_ptr() % 16:
         raise GzkpError(f"{name} must be 16-byte aligned")
@@ -185,13 +207,16 @@ def msm(curve, points, scalars, out=None, stream=None, workspace=None):
     n = P.shape[0]
     if K.shape[0] != n:
         raise GzkpError("points and scalars differ in length")
+    if K.device != P.device:
+        raise GzkpError("points and scalars are on different devices")
     if out is None:
         out = torch.empty(2 * L, dtype=torch.int32, device=P.device)
-    if workspace is None:
-        st = lib().gzkp_msm(cid, P.data_ptr(), K.data_ptr(), n, out.data_ptr(), _stream_ptr(stream))
-    else:
-        st = lib().gzkp_msm_ex(cid, P.data_ptr(), K.data_ptr(), n, out.data_ptr(), workspace.data_ptr(),
-                               workspace.numel() * workspace.element_size(), _stream_ptr(stream))
+    with _on(P):
+        if workspace is None:
+            st = lib().gzkp_msm(cid, P.data_ptr(), K.data_ptr(), n, out.data_ptr(), _stream_ptr(stream, P.device))
+        else:
+            st = lib().gzkp_msm_ex(cid, P.data_ptr(), K.data_ptr(), n, out.data_ptr(), workspace.data_ptr(),
+                                   workspace.numel() * workspace.element_size(), _stream_ptr(stream, P.device))
     _check(st, "gzkp_msm")
     return out
 
@@ -199,10 +224,12 @@ def msm(curve, points, scalars, out=None, stream=None, workspace=None):
 def msm_host(curve, points: np.ndarray, scalars: np.ndarray, out: Optional[np.ndarray] = None, stream=None):
     """MSM from HOST buffers: copies inside the call (the e2e path)."""
     cid = curve_id(curve)
-    L = field_limbs(cid)
-    points = np.ascontiguousarray(points, dtype=np.uint32)
-    scalars = np.ascontiguousarray(scalars, dtype=np.uint32)
-    n = points.shape[0] if points.ndim == 2 else points.size // (2 * L)
+    L, Ls = field_limbs(cid), scalar_limbs(cid)
+    points = _host_u32(points, 2 * L, "points")
+    scalars = _host_u32(scalars, Ls, "scalars")
+    n = points.shape[0]
+    if scalars.shape[0] != n:
+        raise GzkpError("points and scalars differ in length")
     if out is None:
         out = np.zeros(2 * L, dtype=np.uint32)
     st = lib().gzkp_msm_host(cid, points.ctypes.data, scalars.ctypes.data, n, out.ctypes.data, _stream_ptr(stream))
@@ -217,17 +244,20 @@ class PreparedPoints:
         """weighted=None: library default (weighted-point table when it fits);
         True/False force GZKP's cross-window consolidation on/off."""
         self.curve = curve_id(curve)
+        self.handle = None
         L = field_limbs(self.curve)
         P = _dev_u32(points, 2 * L, "points")
         self.n = P.shape[0]
+        self.device = P.device
         h = ctypes.c_void_p()
-        if weighted is None and window_bits == 0:
-            _check(lib().gzkp_points_prepare(self.curve, P.data_ptr(), self.n, ctypes.byref(h), _stream_ptr(stream)),
-                   "gzkp_points_prepare")
-        else:
-            _check(lib().gzkp_points_prepare_ex(self.curve, P.data_ptr(), self.n, window_bits,
-                                                1 if (weighted is None or weighted) else 0, ctypes.byref(h),
-                                                _stream_ptr(stream)), "gzkp_points_prepare_ex")
+        with _on(P):
+            if weighted is None and window_bits == 0:
+                _check(lib().gzkp_points_prepare(self.curve, P.data_ptr(), self.n, ctypes.byref(h),
+                                                 _stream_ptr(stream, P.device)), "gzkp_points_prepare")
+            else:
+                _check(lib().gzkp_points_prepare_ex(self.curve, P.data_ptr(), self.n, window_bits,
+                                                    1 if (weighted is None or weighted) else 0, ctypes.byref(h),
+                                                    _stream_ptr(stream, P.device)), "gzkp_points_prepare_ex")
         self.handle = h
 
     def info(self):
@@ -240,24 +270,33 @@ class PreparedPoints:
         torch = _torch()
         L, Ls = field_limbs(self.curve), scalar_limbs(self.curve)
         K = _dev_u32(scalars, Ls, "scalars")
+        if K.device != self.device:
+            raise GzkpError("scalars must be on the prepared points' device")
+        if K.shape[0] > self.n:
+            raise GzkpError("more scalars than prepared points")
         if out is None:
             out = torch.empty(2 * L, dtype=torch.int32, device=K.device)
-        _check(lib().gzkp_msm_prepared(self.handle, K.data_ptr(), K.shape[0], out.data_ptr(), _stream_ptr(stream)),
-               "gzkp_msm_prepared")
+        with _on(K):
+            _check(lib().gzkp_msm_prepared(self.handle, K.data_ptr(), K.shape[0], out.data_ptr(),
+                                           _stream_ptr(stream, K.device)), "gzkp_msm_prepared")
         return out
 
     def msm_host(self, scalars: np.ndarray, out: Optional[np.ndarray] = None, stream=None):
-        L = field_limbs(self.curve)
-        scalars = np.ascontiguousarray(scalars, dtype=np.uint32)
+        L, Ls = field_limbs(self.curve), scalar_limbs(self.curve)
+        scalars = _host_u32(scalars, Ls, "scalars")
+        if scalars.shape[0] > self.n:
+            raise GzkpError("more scalars than prepared points")
         if out is None:
             out = np.zeros(2 * L, dtype=np.uint32)
-        _check(lib().gzkp_msm_prepared_host(self.handle, scalars.ctypes.data, scalars.shape[0], out.ctypes.data,
-                                            _stream_ptr(stream)), "gzkp_msm_prepared_host")
+        with _torch().cuda.device(self.device):
+            _check(lib().gzkp_msm_prepared_host(self.handle, scalars.ctypes.data, scalars.shape[0], out.ctypes.data,
+                                                _stream_ptr(stream, self.device)), "gzkp_msm_prepared_host")
         return out
 
     def release(self):
-        if self.handle:
-            lib().gzkp_points_release(self.handle)
+        if getattr(self, "handle", None):
+            with _torch().cuda.device(self.device):
+                lib().gzkp_points_release(self.handle)
             self.handle = None
 
     def __del__(self):
@@ -273,10 +312,13 @@ def msm_partial(curve, points, scalars, out=None, stream=None):
     L, Ls = field_limbs(cid), scalar_limbs(cid)
     P = _dev_u32(points, 2 * L, "points")
     K = _dev_u32(scalars, Ls, "scalars")
+    if K.shape[0] != P.shape[0] or K.device != P.device:
+        raise GzkpError("points and scalars differ in length or device")
     if out is None:
         out = torch.empty(4 * L, dtype=torch.int32, device=P.device)
-    _check(lib().gzkp_msm_partial(cid, P.data_ptr(), K.data_ptr(), P.shape[0], out.data_ptr(), _stream_ptr(stream)),
-           "gzkp_msm_partial")
+    with _on(P):
+        _check(lib().gzkp_msm_partial(cid, P.data_ptr(), K.data_ptr(), P.shape[0], out.data_ptr(),
+                                      _stream_ptr(stream, P.device)), "gzkp_msm_partial")
     return out
 
 
@@ -287,8 +329,9 @@ def combine_partials(curve, partials, out=None, stream=None):
     Pt = _dev_u32(partials, 4 * L, "partials")
     if out is None:
         out = torch.empty(2 * L, dtype=torch.int32, device=Pt.device)
-    _check(lib().gzkp_combine_partials(cid, Pt.data_ptr(), Pt.shape[0], out.data_ptr(), _stream_ptr(stream)),
-           "gzkp_combine_partials")
+    with _on(Pt):
+        _check(lib().gzkp_combine_partials(cid, Pt.data_ptr(), Pt.shape[0], out.data_ptr(),
+                                           _stream_ptr(stream, Pt.device)), "gzkp_combine_partials")
     return out
 
 
@@ -300,8 +343,9 @@ def fixed_base_mul(curve, scalars, out=None, stream=None):
     K = _dev_u32(scalars, Ls, "scalars")
     if out is None:
         out = torch.empty((K.shape[0], 2 * L), dtype=torch.int32, device=K.device)
-    _check(lib().gzkp_fixed_base_mul(cid, K.data_ptr(), K.shape[0], out.data_ptr(), _stream_ptr(stream)),
-           "gzkp_fixed_base_mul")
+    with _on(K):
+        _check(lib().gzkp_fixed_base_mul(cid, K.data_ptr(), K.shape[0], out.data_ptr(), _stream_ptr(stream, K.device)),
+               "gzkp_fixed_base_mul")
     return out
 
 
@@ -312,8 +356,9 @@ def field_op(curve, op: int, a, b, stream=None):
     A = _dev_u32(a, L, "a")
     B = _dev_u32(b, L, "b")
     out = torch.empty_like(A)
-    _check(lib().gzkp_field_op(cid, op, A.data_ptr(), B.data_ptr(), out.data_ptr(), A.shape[0], _stream_ptr(stream)),
-           "gzkp_field_op")
+    with _on(A):
+        _check(lib().gzkp_field_op(cid, op, A.data_ptr(), B.data_ptr(), out.data_ptr(), A.shape[0],
+                                   _stream_ptr(stream, A.device)), "gzkp_field_op")
     return out
 
 
@@ -324,8 +369,9 @@ def ec_op(curve, op: int, P, Q, stream=None):
     A = _dev_u32(P, 2 * L, "P")
     B = _dev_u32(Q, 2 * L, "Q")
     out = torch.empty_like(A)
-    _check(lib().gzkp_ec_op(cid, op, A.data_ptr(), B.data_ptr(), out.data_ptr(), A.shape[0], _stream_ptr(stream)),
-           "gzkp_ec_op")
+    with _on(A):
+        _check(lib().gzkp_ec_op(cid, op, A.data_ptr(), B.data_ptr(), out.data_ptr(), A.shape[0],
+                                _stream_ptr(stream, A.device)), "gzkp_ec_op")
     return out
 
 
@@ -349,8 +395,9 @@ def ntt(curve, values, inverse: bool = False, out=None, stream=None):
         raise GzkpError("NTT size must be a power of two")
     if out is None:
         out = torch.empty_like(A)
-    _check(lib().gzkp_ntt(cid, A.data_ptr(), out.data_ptr(), log_n, 1 if inverse else 0, _stream_ptr(stream)),
-           "gzkp_ntt")
+    with _on(A):
+        _check(lib().gzkp_ntt(cid, A.data_ptr(), out.data_ptr(), log_n, 1 if inverse else 0,
+                              _stream_ptr(stream, A.device)), "gzkp_ntt")
     return out
 
 
@@ -366,9 +413,16 @@ def scalar_field_op(curve, op: int, a, b, stream=None):
     A = _dev_u32(a, Ls, "a")
     B = _dev_u32(b, Ls, "b")
     out = torch.empty_like(A)
-    _check(lib().gzkp_scalar_field_op(cid, op, A.data_ptr(), B.data_ptr(), out.data_ptr(), A.shape[0],
-                                      _stream_ptr(stream)), "gzkp_scalar_field_op")
+    with _on(A):
+        _check(lib().gzkp_scalar_field_op(cid, op, A.data_ptr(), B.data_ptr(), out.data_ptr(), A.shape[0],
+                                          _stream_ptr(stream, A.device)), "gzkp_scalar_field_op")
     return out
+
+
+def release_stream(stream=None):
+    """Free the library's cached workspace and side stream for `stream` (call
+    before destroying a stream the library was used on)."""
+    _check(lib().gzkp_release_stream(_stream_ptr(stream)), "gzkp_release_stream")
 
 
 # ------------------------------------------------------------- multi-GPU
@@ -419,10 +473,13 @@ def msm_sharded(curve, points_local, scalars_local, comm: Comm, out=None, stream
     L, Ls = field_limbs(cid), scalar_limbs(cid)
     P = _dev_u32(points_local, 2 * L, "points")
     K = _dev_u32(scalars_local, Ls, "scalars")
+    if K.shape[0] != P.shape[0] or K.device != P.device:
+        raise GzkpError("points and scalars differ in length or device")
     if out is None:
         out = torch.empty(2 * L, dtype=torch.int32, device=P.device)
-    _check(lib().gzkp_msm_sharded(cid, P.data_ptr(), K.data_ptr(), P.shape[0], out.data_ptr(), _stream_ptr(stream),
-                                  comm.handle), "gzkp_msm_sharded")
+    with _on(P):
+        _check(lib().gzkp_msm_sharded(cid, P.data_ptr(), K.data_ptr(), P.shape[0], out.data_ptr(),
+                                      _stream_ptr(stream, P.device), comm.handle), "gzkp_msm_sharded")
     return out
 
 
@@ -431,14 +488,17 @@ def msm_prepared_sharded(prepared: "PreparedPoints", scalars_local, comm: Comm, 
     torch = _torch()
     L, Ls = field_limbs(prepared.curve), scalar_limbs(prepared.curve)
     K = _dev_u32(scalars_local, Ls, "scalars")
+    if K.shape[0] > prepared.n or K.device != prepared.device:
+        raise GzkpError("scalars exceed the prepared shard or are on another device")
     if out is None:
         out = torch.empty(2 * L, dtype=torch.int32, device=K.device)
-    _check(lib().gzkp_msm_prepared_sharded(prepared.handle, K.data_ptr(), K.shape[0], out.data_ptr(),
-                                           _stream_ptr(stream), comm.handle), "gzkp_msm_prepared_sharded")
+    with _on(K):
+        _check(lib().gzkp_msm_prepared_sharded(prepared.handle, K.data_ptr(), K.shape[0], out.data_ptr(),
+                                               _stream_ptr(stream, K.device), comm.handle), "gzkp_msm_prepared_sharded")
     return out
 
 
 __all__ = ["CURVES", "GzkpError", "lib", "msm", "msm_host", "PreparedPoints", "msm_partial", "combine_partials",
            "fixed_base_mul", "field_op", "ec_op", "Comm", "msm_sharded", "msm_prepared_sharded", "shard_range", "set_config",
            "window_bits", "workspace_bytes", "set_profiling", "profile_read", "field_limbs", "scalar_limbs", "to_device",
-           "to_numpy", "ntt", "ntt_max_log", "ntt_last_launches", "scalar_field_op"]
+           "to_numpy", "ntt", "ntt_max_log", "ntt_last_launches", "scalar_field_op", "release_stream"]

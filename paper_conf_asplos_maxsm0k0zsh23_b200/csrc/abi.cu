@@ -13,7 +13,9 @@
 #include <cstring>
 #include <map>
 #include <mutex>
+#include <set>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "internal.h"
@@ -102,42 +104,100 @@ const CurveImpl* impl_for(int curve) {
   }
 }
 
-// the stream-ordered pool keeps freed workspace (no re-allocation per call)
+int current_device() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  return dev;
+}
+
+gzkp_status once_per_device(const void* key, const std::function<gzkp_status()>& f) {
+  static std::mutex mu;
+  static std::set<std::pair<int, const void*>> done;
+  const std::pair<int, const void*> k{current_device(), key};
+  std::lock_guard<std::mutex> lock(mu);
+  if (done.count(k)) return GZKP_SUCCESS;
+  gzkp_status st = f();
+  if (st == GZKP_SUCCESS) done.insert(k);
+  return st;
+}
+
+static std::mutex g_pool_mu;
+static std::map<int, cudaMemPool_t> g_pools;
+
+static cudaMemPool_t device_pool(int dev) {
+  std::lock_guard<std::mutex> lock(g_pool_mu);
+  auto it = g_pools.find(dev);
+  return it == g_pools.end() ? nullptr : it->second;
+}
+
+// per device: the library's private stream-ordered pool (freed workspace is
+// kept for the next call without changing the application's default pool)
+// and the call-stack limit of the out-of-line MNT4-753 paths (~2.6 KB per
+// thread, ptxas "cumulative stack size"; the default limit is 1 KB)
 void init_pool_once() {
-  static std::once_flag once;
-  std::call_once(once, [] {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+  static int tag;
+  once_per_device(&tag, [] {
+    const int dev = current_device();
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t pool = nullptr;
+    if (cudaMemPoolCreate(&pool, &props) == cudaSuccess) {
       uint64_t thr = UINT64_MAX;
       cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+      std::lock_guard<std::mutex> lock(g_pool_mu);
+      g_pools[dev] = pool;
     }
-    // the out-of-line MNT4-753 paths need up to ~2.6 KB of call stack per
-    // thread (ptxas "cumulative stack size"); the default limit is 1 KB
+    cudaGetLastError();
     size_t stack = 0;
     cudaDeviceGetLimit(&stack, cudaLimitStackSize);
     if (stack < 4096) cudaDeviceSetLimit(cudaLimitStackSize, 4096);
+    return GZKP_SUCCESS;
   });
+}
+
+cudaError_t pool_malloc(void** p, size_t bytes, cudaStream_t s) {
+  cudaMemPool_t pool = device_pool(current_device());
+  return pool ? cudaMallocFromPoolAsync(p, bytes, pool, s) : cudaMallocAsync(p, bytes, s);
 }
 
 static bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 
+// Per-stream library state, keyed by (device, stream handle, thread): calls
+// on one stream are ordered, so they can share a workspace; different streams
+// never do.  cudaStreamPerThread is one handle for many per-thread streams, so
+// it is keyed by the calling thread as well.  gzkp_release_stream drops the
+// entries of a stream before the application destroys it.
+struct StreamKey {
+  int dev;
+  cudaStream_t s;
+  size_t tid;
+  bool operator<(const StreamKey& o) const {
+    return dev != o.dev ? dev < o.dev : s != o.s ? s < o.s : tid < o.tid;
+  }
+};
+static StreamKey stream_key(cudaStream_t s) {
+  size_t tid = 0;
+  if (s == cudaStreamPerThread) tid = std::hash<std::thread::id>{}(std::this_thread::get_id());
+  return {current_device(), s, tid};
+}
+struct WsEntry { void* p; size_t bytes; };
+static std::mutex g_ws_mu;
+static std::map<StreamKey, WsEntry> g_ws;
+static std::mutex g_ctx_mu;
+static std::map<StreamKey, StreamCtx*> g_ctx;
+
 gzkp_status stream_workspace(cudaStream_t s, size_t bytes, void** ptr) {
-  struct Entry { void* p; size_t bytes; };
-  static std::mutex mu;
-  static std::map<std::pair<int, cudaStream_t>, Entry> cache;
-  int dev = 0;
-  cudaGetDevice(&dev);
-  std::lock_guard<std::mutex> lock(mu);
-  Entry& e = cache[{dev, s}];
+  std::lock_guard<std::mutex> lock(g_ws_mu);
+  WsEntry& e = g_ws[stream_key(s)];
   if (e.bytes < bytes) {
     // stream-ordered: the old buffer is released after the work already queued on s
     if (e.p) cudaFreeAsync(e.p, s);
     e.p = nullptr;
     e.bytes = 0;
     const size_t want = bytes + bytes / 8;   // headroom against small n changes
-    cudaError_t err = cudaMallocAsync(&e.p, want, s);
+    cudaError_t err = pool_malloc(&e.p, want, s);
     if (err != cudaSuccess) {
       e.p = nullptr;
       return cuda_status(err, "cudaMallocAsync(workspace)");
@@ -149,12 +209,8 @@ gzkp_status stream_workspace(cudaStream_t s, size_t bytes, void** ptr) {
 }
 
 gzkp_status stream_ctx(cudaStream_t s, StreamCtx** out) {
-  static std::mutex mu;
-  static std::map<std::pair<int, cudaStream_t>, StreamCtx*> cache;
-  int dev = 0;
-  cudaGetDevice(&dev);
-  std::lock_guard<std::mutex> lock(mu);
-  StreamCtx*& c = cache[{dev, s}];
+  std::lock_guard<std::mutex> lock(g_ctx_mu);
+  StreamCtx*& c = g_ctx[stream_key(s)];
   if (!c) {
     StreamCtx* n = new StreamCtx;
     int lo = 0, hi = 0;
@@ -167,6 +223,31 @@ gzkp_status stream_ctx(cudaStream_t s, StreamCtx** out) {
   }
   *out = c;
   return GZKP_SUCCESS;
+}
+
+// frees the workspace (stream-ordered) and the side stream of (device, s)
+static gzkp_status release_stream(cudaStream_t s) {
+  const StreamKey k = stream_key(s);
+  {
+    std::lock_guard<std::mutex> lock(g_ws_mu);
+    auto it = g_ws.find(k);
+    if (it != g_ws.end()) {
+      if (it->second.p) cudaFreeAsync(it->second.p, s);
+      g_ws.erase(it);
+    }
+  }
+  std::lock_guard<std::mutex> lock(g_ctx_mu);
+  auto it = g_ctx.find(k);
+  if (it != g_ctx.end()) {
+    StreamCtx* c = it->second;
+    cudaStreamSynchronize(c->side);
+    for (int i = 0; i < c->nev; ++i) cudaEventDestroy(c->ev[i]);
+    cudaStreamDestroy(c->side);
+    delete c;
+    g_ctx.erase(it);
+  }
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? GZKP_SUCCESS : cuda_status(e, "gzkp_release_stream");
 }
 
 struct Prepared {
@@ -329,7 +410,7 @@ gzkp_status gzkp_msm_host(int curve, const void* points_host, const void* scalar
   // staging (canonical points as copied), Montgomery points, scalars, out
   char* d = nullptr;
   const size_t total = 2 * align_up(pb) + align_up(sb) + align_up(ob);
-  cudaError_t e = cudaMallocAsync((void**)&d, total, s);
+  cudaError_t e = pool_malloc((void**)&d, total, s);
   if (e != cudaSuccess) return cuda_status(e, "cudaMallocAsync");
   char *dstage = d, *dp = d + align_up(pb), *ds = d + 2 * align_up(pb), *dout = ds + align_up(sb);
   gzkp_status st = GZKP_SUCCESS;
@@ -379,6 +460,10 @@ gzkp_status gzkp_points_prepare_ex(int curve, const void* points_affine, size_t 
   if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
   if (!handle || (n && !points_affine) || !aligned16(points_affine) || window_bits < 0 || window_bits > 22)
     return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
+  // the standard (per-window bucket sets) pipeline plans c <= 16, as gzkp_set_config
+  if (weighted != 1 && (window_bits == 1 || window_bits > 16))
+    return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..16 for unweighted points");
+  if (weighted == 1 && window_bits == 1) return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..22");
   Prepared* h = new (std::nothrow) Prepared{curve, n, nullptr, false, 0, 1, 0};
   if (!h) return set_error(GZKP_ERROR_OUT_OF_MEMORY, "handle");
   const size_t pt_bytes = 2 * (size_t)c->limbs * 4;
@@ -459,7 +544,7 @@ gzkp_status gzkp_msm_prepared_host(const void* handle, const void* scalars_host,
   cudaStream_t s = (cudaStream_t)stream;
   const size_t sb = n * c->scalar_limbs * 4, ob = 2 * c->limbs * 4;
   char* d = nullptr;
-  cudaError_t e = cudaMallocAsync((void**)&d, align_up(sb) + align_up(ob), s);
+  cudaError_t e = pool_malloc((void**)&d, align_up(sb) + align_up(ob), s);
   if (e != cudaSuccess) return cuda_status(e, "cudaMallocAsync");
   void *ds = d, *dout = d + align_up(sb);
   gzkp_status st = GZKP_SUCCESS;
@@ -629,6 +714,8 @@ gzkp_status gzkp_msm_prepared_sharded(const void* handle, const void* scalars, s
     return st;
   return c->combine(cm->gathered, cm->world, out, s);
 }
+
+gzkp_status gzkp_release_stream(gzkp_stream stream) { return release_stream((cudaStream_t)stream); }
 
 const char* gzkp_status_string(gzkp_status status) {
   switch (status) {

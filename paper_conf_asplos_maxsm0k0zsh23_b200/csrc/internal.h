@@ -5,6 +5,7 @@
 
 #include <cstddef>
 #include <cstdint>
+#include <functional>
 #include <string>
 #include <vector>
 
@@ -94,8 +95,17 @@ struct StreamCtx {
   int nev = 0;
 };
 gzkp_status stream_ctx(cudaStream_t s, StreamCtx** ctx);
-// once per process: stream-ordered pool release threshold, and a 4 KB
-// per-thread stack for the out-of-line MNT4-753 products (every entry point)
+// once per DEVICE (every entry point calls it for the current device): the
+// library's private stream-ordered memory pool (release threshold = max, so
+// freed workspace is kept; the device's default pool is left untouched) and a
+// 4 KB per-thread stack for the out-of-line MNT4-753 products.
 void init_pool_once();
+// Runs f() once per (key, current device), under a process-wide lock;
+// per-device state (kernel attributes, limits) must never hide behind a
+// process-wide flag.  A failing f() is retried by the next call.
+gzkp_status once_per_device(const void* key, const std::function<gzkp_status()>& f);
+int current_device();
+// stream-ordered allocation from the library's private pool of the current device
+cudaError_t pool_malloc(void** p, size_t bytes, cudaStream_t s);
 
 }  // namespace gzkp

@@ -8,6 +8,8 @@
 #pragma once
 #include <cmath>
 #include <cstdlib>
+#include <map>
+#include <mutex>
 #include <vector>
 
 #include "internal.h"
@@ -123,15 +125,21 @@ struct Impl {
   // so S in [40, 64] is picked to make the wave count just below an integer
   // (E estimated as n W, exact for uniform scalars up to zero digits).
   static uint64_t accum_resident_threads() {
-    static const uint64_t v = [] {
-      int per_sm = 0;
-      const size_t smem = (size_t)128 * Stage<C>::SLOT_WORDS * 4;
-      if (smem > 48 * 1024 ||
-          cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_accum<C>, 128, smem) != cudaSuccess)
-        per_sm = 0;
-      cudaGetLastError();
-      return (uint64_t)per_sm * device_sm_count() * 128;
-    }();
+    // per device (a multi-GPU process may drive GPUs of different SM counts)
+    static std::mutex mu;
+    static std::map<int, uint64_t> cache;
+    const int dev = current_device();
+    std::lock_guard<std::mutex> lock(mu);
+    auto it = cache.find(dev);
+    if (it != cache.end()) return it->second;
+    int per_sm = 0;
+    const size_t smem = (size_t)128 * Stage<C>::SLOT_WORDS * 4;
+    if (smem > 48 * 1024 ||
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_accum<C>, 128, smem) != cudaSuccess)
+      per_sm = 0;
+    cudaGetLastError();
+    const uint64_t v = (uint64_t)per_sm * device_sm_count() * 128;
+    cache[dev] = v;
     return v;
   }
   static int chunk_entries_for(uint64_t E) {
@@ -292,6 +300,9 @@ struct Impl {
     if ((uint64_t)n >= (1ull << 31)) return set_error(GZKP_ERROR_INVALID_VALUE, "n >= 2^31 not supported");
     const Plan p = plan(n, call.prepared, call.consolidated, call.window_bits, call.table_n);
     if (p.E_max >= (1ull << 32) - 1) return set_error(GZKP_ERROR_INVALID_VALUE, "n * windows >= 2^32");
+    // the bucket-offset scan is two-level: <= SCAN_TILE tiles of SCAN_TILE keys
+    if ((uint64_t)p.M > (uint64_t)SCAN_TILE * SCAN_TILE)
+      return set_error(GZKP_ERROR_INVALID_VALUE, "too many bucket keys (window bits too large for this curve)");
     if (p.consolidated && (uint64_t)p.val_stride * p.W >= (1ull << 31))
       return set_error(GZKP_ERROR_INVALID_VALUE, "weighted-point table >= 2^31 points");
     char* ws = (char*)call.workspace;
@@ -375,22 +386,23 @@ struct Impl {
       const char* e = getenv("GZKP_ACCUM_MINB");
       return AccumCfg<C>::DFP && e && atoi(e) == 3;
     }();
-    static bool attr_set = false;
-    if (!attr_set) {
-      GZ_CHECK(cudaFuncSetAttribute(k_accum<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
-      if constexpr (AccumCfg<C>::DFP)
-        GZ_CHECK(cudaFuncSetAttribute(k_accum<C, false, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
-      if constexpr (AccumCfg<C>::DFP)
-        GZ_CHECK(cudaFuncSetAttribute(k_accum<C, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                      (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
-      GZ_CHECK(cudaFuncSetAttribute(k_reduce_bits<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    (int)((size_t)RB_THREADS * 4 * N * 4)));
-      GZ_CHECK(cudaFuncSetAttribute(k_heavy_tree<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    (int)((size_t)HEAVY_THREADS * 4 * N * 4)));
-      attr_set = true;
-    }
+    static int attr_tag;   // kernel attributes are per device
+    if (gzkp_status st = once_per_device(&attr_tag, [] {
+          GZ_CHECK(cudaFuncSetAttribute(k_accum<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
+          if constexpr (AccumCfg<C>::DFP)
+            GZ_CHECK(cudaFuncSetAttribute(k_accum<C, false, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
+          if constexpr (AccumCfg<C>::DFP)
+            GZ_CHECK(cudaFuncSetAttribute(k_accum<C, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
+          GZ_CHECK(cudaFuncSetAttribute(k_reduce_bits<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        (int)((size_t)RB_THREADS * 4 * N * 4)));
+          GZ_CHECK(cudaFuncSetAttribute(k_heavy_tree<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        (int)((size_t)HEAVY_THREADS * 4 * N * 4)));
+          return GZKP_SUCCESS;
+        }))
+      return st;
     // overlapped host->device path: the points are still arriving on another
     // stream while the digits / sort ran; only the accumulation needs them
     if (call.points_ready) GZ_CHECK(cudaStreamWaitEvent(s, call.points_ready, 0));

@@ -53,7 +53,10 @@ struct NttImpl {
       const int grid = (int)std::max<uint64_t>(1, std::min<uint64_t>((work + threads - 1) / threads,
                                                                      (uint64_t)device_sm_count() * 8));
       k_ntt_twiddles<R><<<grid, threads, 0, s>>>(t.tw, t.half, log_n, inverse, t.tw + t.half * L);
+      // publish the table only once it is built: a later call on another
+      // (non-blocking) stream must never read it half-written
       cudaError_t e = cudaGetLastError();
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s);
       if (e != cudaSuccess) {
         cudaFree(t.tw);
         t.tw = nullptr;
@@ -69,7 +72,6 @@ struct NttImpl {
     const size_t bytes = n * L * 4;
     NttTables* tb = nullptr;
     if (gzkp_status st = tables(fid, log_n, inverse, s, &tb)) return st;
-    static bool attr = false;
     const size_t smem = ((size_t)1 << TILE_LOG) * L * 4;
     // register budget: MIN_CTAS CTAs/SM (the shared-memory limit) or, with
     // GZKP_NTT_MINB=2 (8-limb fields), 2 CTAs/SM with up to 128 registers
@@ -78,11 +80,13 @@ struct NttImpl {
       return L <= 8 && e && atoi(e) == 2;
     }();
     auto kern = two ? k_ntt_pass<R, 2> : k_ntt_pass<R>;
-    if (!attr) {
-      NTT_CHECK(cudaFuncSetAttribute(k_ntt_pass<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      NTT_CHECK(cudaFuncSetAttribute(k_ntt_pass<R, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-      attr = true;
-    }
+    static int attr_tag;   // per device
+    if (gzkp_status st = once_per_device(&attr_tag, [smem] {
+          NTT_CHECK(cudaFuncSetAttribute(k_ntt_pass<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+          NTT_CHECK(cudaFuncSetAttribute(k_ntt_pass<R, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+          return GZKP_SUCCESS;
+        }))
+      return st;
     *launches = 0;
     if (log_n == 0) {   // N = 1: a_0 = A_0 (N^-1 = 1)
       if (in != out) NTT_CHECK(cudaMemcpyAsync(out, in, bytes, cudaMemcpyDeviceToDevice, s));
