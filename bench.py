@@ -47,6 +47,7 @@ WORKLOADS = {
     "bn254_2p10": ("bn254", 10, 1, "uniform", "BN254 G1 MSM n=2^10, uniform random scalars"),
     # one rank's shard of configs[2] at 8 GPUs (diagnostic: the per-GPU step of the 8-GPU run)
     "bls12_381_2p19": ("bls12_381", 19, 3, "uniform", "BLS12-381 G1 MSM n=2^19 (one rank's shard of n=2^22 at 8 GPUs)"),
+    "mnt4_753_2p17": ("mnt4_753", 17, 4, "uniform", "MNT4-753 G1 MSM n=2^17 (one rank's shard of n=2^20 at 8 GPUs)"),
     # G2 (not a BASELINE config: the same MSM over F_p^2)
     "bn254_g2_2p20": ("bn254_g2", 20, 7, "uniform", "BN254 G2 MSM n=2^20, uniform scalars (NEXT-3)"),
     "bls12_381_g2_2p20": ("bls12_381_g2", 20, 8, "uniform", "BLS12-381 G2 MSM n=2^20, uniform scalars (NEXT-3)"),
@@ -141,6 +142,20 @@ class ClockSampler:
             return None
         return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(smax), "reasons": sorted(reasons),
                 "samples": len(sm)}
+
+
+def relaunch_distributed(nproc: int) -> int:
+    """`python bench.py --gpus N` without a launcher: re-run this command under
+    torch.distributed.run with N ranks on this node (one per GPU, rendezvous on
+    127.0.0.1), exactly as the driver launches it; rank 0 prints the line."""
+    import socket
+    sock = socket.socket()
+    sock.bind(("127.0.0.1", 0))
+    port = sock.getsockname()[1]
+    sock.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 def dist_env():
@@ -387,6 +402,15 @@ def main():
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
     wl = args.workload
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(relaunch_distributed(args.gpus))
+    if "WORLD_SIZE" in os.environ and int(os.environ["WORLD_SIZE"]) != args.gpus:
+        sys.exit(f"bench.py: WORLD_SIZE={os.environ['WORLD_SIZE']} but --gpus {args.gpus}")
+    if int(os.environ.get("WORLD_SIZE", "1")) > 1:
+        # the communicator set-up log (one "comm ... rank r nranks N" line per
+        # rank) shows which ranks and transports the collective really used
+        os.environ.setdefault("NCCL_DEBUG", "INFO")
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
 
     if wl in NTT_WORKLOADS:
         if args.impl == "reference":
@@ -424,8 +448,9 @@ def main():
     n_loc = hi - lo
 
     # ---- inputs (seeded; points generated on the device) ----
-    dl = synth.dlogs(curve, n, synth.dlog_seed(curve))[lo:hi]
-    ks = synth.scalars(curve, n, synth.scalar_seed(cfg), sdist)[lo:hi]
+    dl_full = synth.dlogs(curve, n, synth.dlog_seed(curve))
+    ks_full = synth.scalars(curve, n, synth.scalar_seed(cfg), sdist)
+    dl, ks = dl_full[lo:hi], ks_full[lo:hi]
     P = torch.empty((n_loc, 2 * L), dtype=torch.int32, device="cuda")
     step_gen = 1 << 20
     for s0 in range(0, n_loc, step_gen):
@@ -497,6 +522,7 @@ def main():
     clocks = sampler.stop()
     prof = gz.profile_read(reset=True)
     gz.set_profiling(False)
+    result = gz.to_numpy(out).copy()          # the timed steps' MSM value (parity leg below)
 
     t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
     if world > 1:
@@ -504,37 +530,69 @@ def main():
     total_ms = float(t.item())
 
     # ---- the same MSM on prepared weighted points (GZKP cross-window
-    # consolidation): setup-time table, timed like the above
+    # consolidation): setup-time table per rank (its shard),
+    # timed like the above (max over ranks); N > 1 through the same one
+    # all-gather (gzkp_msm_prepared_sharded)
     prepared = None
-    if world == 1 and not args.no_prepared:
+    if not args.no_prepared:
         t0 = time.perf_counter()
         hp = gz.PreparedPoints(curve, P, weighted=True)
         torch.cuda.synchronize()
         prep_s = time.perf_counter() - t0
         info = hp.info()
+
+        pout = torch.empty_like(out)
+
+        def pstep():
+            if comm is None:
+                hp.msm(K, out=pout)
+            else:
+                gz.msm_prepared_sharded(hp, K, comm, out=pout)
+
         for _ in range(args.warmup):
-            hp.msm(K, out=out)
+            pstep()
         torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
         gz.set_profiling(True)
         gz.profile_read(reset=True)
         pe0, pe1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         pe0.record(stream)
         for _ in range(args.steps):
-            hp.msm(K, out=out)
+            pstep()
         pe1.record(stream)
         torch.cuda.synchronize()
         pprof = gz.profile_read(reset=True)
         gz.set_profiling(False)
-        p_ms = pe0.elapsed_time(pe1) / args.steps
+        presult = gz.to_numpy(pout).copy()
+        tp = torch.tensor([pe0.elapsed_time(pe1)], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(tp, op=dist.ReduceOp.MAX)
+        p_ms = float(tp.item()) / args.steps
         pcalls = max(1, pprof["calls"])
         p_accum = pprof["phase_ms"]["accumulate"] / pcalls
         p_ach = pprof["entries"] * madd_imad(L, g2) / (p_accum / 1e3) if p_accum > 0 else 0.0
         prepared = {"value": n / (p_ms / 1e3), "unit": "points/s", "ms_per_step": p_ms,
                     "window_bits": info["window_bits"], "windows": info["windows"],
-                    "table_bytes": info["bytes"], "prepare_s": prep_s,
+                    "table_bytes_per_gpu": info["bytes"], "prepare_s": prep_s,
                     "accum_frac_imad_peak": p_ach / (148 * 64 * float(load_peaks()[0].get("sm_max_mhz", 1965.0)) * 1e6),
                     "phase_ms_per_step": {k: round(v / pcalls, 4) for k, v in pprof["phase_ms"].items()},
-                    "api": "gzkp_points_prepare (weighted table, setup) + gzkp_msm_prepared (timed)"}
+                    "api": "gzkp_points_prepare (weighted table, setup) + "
+                           + ("gzkp_msm_prepared" if comm is None else "gzkp_msm_prepared_sharded") + " (timed)"}
+        # fixed-key end to end (the proving key stays resident):
+        # scalars H2D + MSM + result D2H through gzkp_msm_prepared_host
+        if world == 1 and not args.no_e2e:
+            kn = K.cpu().pin_memory().numpy().view(np.uint32)
+            outh = np.zeros(2 * L, dtype=np.uint32)
+            hp.msm_host(kn, outh)
+            k_e2e = max(1, min(args.steps, 5))
+            t0 = time.perf_counter()
+            for _ in range(k_e2e):
+                hp.msm_host(kn, outh)
+            pe2e_ms = (time.perf_counter() - t0) * 1e3 / k_e2e
+            prepared["e2e"] = {"value": n / (pe2e_ms / 1e3), "unit": "points/s", "ms_per_step": pe2e_ms,
+                               "h2d_bytes_per_step": int(K.numel() * 4), "d2h_bytes_per_step": 2 * L * 4,
+                               "api": "gzkp_msm_prepared_host (points resident, scalars from pinned host memory)"}
         hp.release()
         del hp
     ms_per_step = total_ms / args.steps
@@ -603,18 +661,30 @@ def main():
                "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world,
                "api": "gzkp_msm_host" if world == 1 else "H2D + gzkp_msm_sharded + D2H"}
 
-    # ---- cpu baseline: the oracle on a bounded sample (rank 0, N = 1 only) ----
+    # ---- cpu baseline + parity leg (the only place the GPU arm runs the
+    # oracle, after every timed region): the oracle timed on a bounded sample
+    # (rank 0, N = 1), and the full-size result checked against the oracle's
+    # closed form (sum k_i a_i mod r) G (rank 0, every N) ----
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    parity = None
+    if rank == 0 and not args.no_cpu_baseline:
         import oracle
-        n_s = min(n, calibrate_oracle_n(curve, 12.0))
-        rate, wall, cores, spts, sk, sout = oracle_time_sample(curve, n_s, cfg, sdist, 12.0)
-        gout = gz.to_numpy(gz.msm(curve, gz.to_device(spts), gz.to_device(sk)))
-        cpu = {"value": rate, "unit": "points/s", "cores": cores, "kind": "oracle",
-               "sample": f"{n_s} points of {wl} (scalars = the workload's first {n_s}; points tiled "
-                         f"from {min(n_s, max(8, 16 * cores))} oracle a_i*G), wall {wall:.1f} s",
-               "sample_parity_gpu_vs_oracle": bool(np.array_equal(gout, sout))}
+        if world == 1:
+            n_s = min(n, calibrate_oracle_n(curve, 12.0))
+            rate, wall, cores, spts, sk, sout = oracle_time_sample(curve, n_s, cfg, sdist, 12.0)
+            gout = gz.to_numpy(gz.msm(curve, gz.to_device(spts), gz.to_device(sk)))
+            cpu = {"value": rate, "unit": "points/s", "cores": cores, "kind": "oracle",
+                   "sample": f"{n_s} points of {wl} (scalars = the workload's first {n_s}; points tiled "
+                             f"from {min(n_s, max(8, 16 * cores))} oracle a_i*G), wall {wall:.1f} s",
+                   "sample_parity_gpu_vs_oracle": bool(np.array_equal(gout, sout))}
+        t0 = time.perf_counter()
+        want = oracle.closed_form(curve, ks_full, dl_full)
+        parity = {"check": "timed MSM bytes == oracle closed form (sum_i k_i a_i mod r) G at full n",
+                  "ok": bool(np.array_equal(result, want)),
+                  "prepared_ok": None if prepared is None else bool(np.array_equal(presult, want)),
+                  "oracle_s": round(time.perf_counter() - t0, 1)}
 
+    line = None
     if rank == 0:
         line = {
             "metric": metric_for(curve), "value": value, "unit": "points/s", "n_gpus": world, "steps": args.steps,
@@ -624,14 +694,17 @@ def main():
             "config": {"workload": wl, "curve": curve, "n": n, "scalars": sdist, "baseline_config": desc,
                        "window_bits": int(prof["c"]), "parallelism": f"shard{world}" if world > 1 else "single",
                        "l2": "flushed between steps" if flush_l2 else f"inputs {input_bytes >> 20} MiB/GPU > L2"},
-            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "clocks": clocks, "prepared": prepared,
-            "gpu_launches": launches * args.steps, "step_ms": step_ms,
+            "roofline": roofline, "cpu_baseline": cpu, "parity": parity, "e2e": e2e, "clocks": clocks,
+            "prepared": prepared, "gpu_launches": launches * args.steps, "step_ms": step_ms,
         }
-        print(json.dumps(line), flush=True)
     if comm is not None:
         comm.destroy()
     if world > 1:
+        dist.barrier()
         dist.destroy_process_group()
+    if line is not None:
+        # printed last, after the communicators' teardown logs
+        print(json.dumps(line), flush=True)
 
 
 if __name__ == "__main__":

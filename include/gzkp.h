@@ -38,8 +38,12 @@
  * ERRORS: argument errors are reported synchronously (NULL with n > 0,
  * misalignment, unknown curve).  n == 0 writes (0,0).  Kernel faults surface as
  * GZKP_ERROR_CUDA from a later call or a stream synchronisation.  Inputs are
- * not validated (on-curve, < p) unless GZKP_DEBUG_CHECKS=1.  No exception
- * crosses the ABI; gzkp_last_error() gives thread-local detail.
+ * not validated unless the environment sets GZKP_DEBUG_CHECKS=1: then every
+ * MSM / prepare entry point first checks, on the device, that each point is
+ * (0,0) or has canonical coordinates (< p) satisfying y^2 = x^3 + a x + b,
+ * and that each scalar is < 2^b, synchronises `stream`, and returns
+ * GZKP_ERROR_INVALID_VALUE (detail in gzkp_last_error) before any MSM work.
+ * No exception crosses the ABI; gzkp_last_error() gives thread-local detail.
  *
  * THREADING: calls on different streams are independent (each call owns its
  * workspace).  Two concurrent gzkp_msm_sharded calls on one communicator are
@@ -183,6 +187,18 @@ gzkp_status gzkp_fixed_base_mul(int curve, const void *scalars, size_t n, void *
                                 gzkp_stream stream);
 
 /* --- diagnostics ----------------------------------------------------------- */
+/* Test hook (not on the MSM path): runs ONLY the product's digit + sort stage
+ * (a2-a3: signed c-bit windows, §2.3 / Figure 3; the bucket
+ * layout p_index of PAPER.md:206) for `scalars` (device, n x scalar_bytes) at
+ * window bits c in 2..16, synchronises, and copies to HOST memory:
+ *   offsets_host[0 .. W 2^(c-1)]: bucket key t 2^(c-1) + |d| - 1 (window t,
+ *     digit d != 0) owns entries [offsets[key], offsets[key+1]);
+ *   vals_host[0 .. E): point index | 0x80000000 if the digit is negative,
+ *     E = offsets[W 2^(c-1)].  The order inside a bucket is unspecified.
+ * offsets_cap / vals_cap are the buffers' capacities in u32 words. */
+gzkp_status gzkp_debug_buckets(int curve, const void *scalars, size_t n, int window_bits,
+                               uint32_t *offsets_host, size_t offsets_cap, uint32_t *vals_host,
+                               size_t vals_cap, gzkp_stream stream);
 /* Elementwise field ops on canonical inputs (device arrays of n elements):
  * op 0: a*b mod p, 1: a+b, 2: a-b, 3: a^-1 (a != 0), 4: round trip to/from Montgomery,
  * 5: a^2 mod p (the dedicated Montgomery squaring), 6: a*b mod p by the FP64

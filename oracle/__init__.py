@@ -220,8 +220,8 @@ def poly_eval(curve, coeffs: np.ndarray, xs, nthreads: int | None = None) -> lis
 def closed_form(curve, scalars: np.ndarray, dlogs: np.ndarray) -> np.ndarray:
     """sum_i k_i (a_i G) = (sum_i k_i a_i mod r) G  (SURVEY.md §8(c) pins).
 
-    The exact integer sum_i k_i a_i is computed with 16-bit limbs so that every
-    numpy partial sum stays below 2^64 (each product < 2^32, n < 2^31)."""
+    dlogs may hold fewer rows m than there are scalars: a_i = dlogs[i mod m]
+    (the tiled point sets P_i = T[i mod m] of SURVEY.md §8(d))."""
     c = get(curve)
     s = dot_mod(scalars, dlogs, c.r)
     Ls = c.scalar_limbs
@@ -229,23 +229,44 @@ def closed_form(curve, scalars: np.ndarray, dlogs: np.ndarray) -> np.ndarray:
     return mul_each(c, generator_limbs(c), k, 1)[0]
 
 
-def dot_mod(scalars: np.ndarray, dlogs: np.ndarray, r: int) -> int:
-    """(sum_i k_i a_i) mod r, exactly, for u32-limb arrays."""
-    k16 = _u32(scalars).view(np.uint16).astype(np.uint64)   # little-endian halves
-    a16 = _u32(dlogs).view(np.uint16).astype(np.uint64)
-    n = k16.shape[0]
-    if n >= (1 << 31):
-        raise ValueError("n too large for exact 16-bit accumulation")
+def dot_mod(scalars: np.ndarray, dlogs: np.ndarray, r: int, chunk: int = 1 << 20) -> int:
+    """(sum_i k_i a_{i mod m}) mod r, exactly, for u32-limb arrays (m = rows
+    of dlogs).
+
+    Both operands are split into 16-bit limbs and M[u, v] = sum_i k16[i, u]
+    a16[i, v] is formed per chunk of <= 2^20 rows as a float64 matrix product:
+    every product is < 2^32 and a chunk's sum < 2^52, so the float64 values
+    are exact integers.  The chunks' matrices are added as Python ints, then
+    total = sum_{u,v} M[u, v] 2^(16 (u + v))."""
+    if chunk > (1 << 20):
+        raise ValueError("chunk too large for exact float64 accumulation")
+    scalars = _u32(scalars)
+    dlogs = _u32(dlogs)
+    n = scalars.shape[0]
+    m = dlogs.shape[0]
+    if n == 0:
+        return 0
+    if m == 0:
+        raise ValueError("no discrete logs")
+    a16_all = dlogs.view(np.uint16).astype(np.float64)           # [m, 2 La] little-endian halves
+    acc = None
+    for s0 in range(0, n, chunk):
+        s1 = min(n, s0 + chunk)
+        k16 = scalars[s0:s1].view(np.uint16).astype(np.float64)
+        idx = np.arange(s0, s1) % m
+        M = k16.T @ a16_all[idx]
+        Mi = [[int(x) for x in row] for row in M]
+        if acc is None:
+            acc = Mi
+        else:
+            for u in range(len(acc)):
+                for v in range(len(acc[u])):
+                    acc[u][v] += Mi[u][v]
     total = 0
-    # M[u, v] = sum_i k16[i,u] * a16[i,v]  (exact in uint64)
-    step = 1 << 20
-    for s0 in range(0, n, step):
-        M = k16[s0:s0 + step].T @ a16[s0:s0 + step]
-        for u in range(M.shape[0]):
-            for v in range(M.shape[1]):
-                m = int(M[u, v])
-                if m:
-                    total += m << (16 * (u + v))
+    for u, row in enumerate(acc):
+        for v, x in enumerate(row):
+            if x:
+                total += x << (16 * (u + v))
     return total % r
 
 

@@ -79,6 +79,8 @@ def lib():
             "gzkp_ntt_last_launches": ([], i32),
             "gzkp_scalar_field_op": ([i32, i32, vp, vp, vp, sz, vp], i32),
             "gzkp_release_stream": ([vp], i32),
+            "gzkp_debug_buckets": ([i32, vp, sz, i32, ctypes.POINTER(ctypes.c_uint32), sz,
+                                    ctypes.POINTER(ctypes.c_uint32), sz, vp], i32),
             "gzkp_status_string": ([i32], ctypes.c_char_p),
             "gzkp_last_error": ([], ctypes.c_char_p),
         }
@@ -419,6 +421,28 @@ def scalar_field_op(curve, op: int, a, b, stream=None):
     return out
 
 
+def debug_buckets(curve, scalars, window_bits: int, stream=None):
+    """Test hook: the product's digit + sort stage alone (gzkp_debug_buckets).
+    Returns (offsets [W 2^(c-1) + 1], vals [E]) as u32 numpy arrays: bucket
+    key t 2^(c-1) + |d| - 1 owns vals[offsets[key]:offsets[key+1]], each
+    val = point index | 0x80000000 for a negative digit."""
+    cid = curve_id(curve)
+    Ls = scalar_limbs(cid)
+    K = _dev_u32(scalars, Ls, "scalars")
+    n = K.shape[0]
+    sbits = {0: 254, 1: 255, 2: 753, 3: 254, 4: 255, 100: 14, 101: 14}[cid]
+    W = -(-(sbits + 1) // window_bits)
+    M = W << (window_bits - 1)
+    off = np.zeros(M + 1, dtype=np.uint32)
+    vals = np.zeros(max(1, n * W), dtype=np.uint32)
+    u32p = ctypes.POINTER(ctypes.c_uint32)
+    with _on(K):
+        _check(lib().gzkp_debug_buckets(cid, K.data_ptr(), n, window_bits, off.ctypes.data_as(u32p), off.size,
+                                        vals.ctypes.data_as(u32p), vals.size, _stream_ptr(stream, K.device)),
+               "gzkp_debug_buckets")
+    return off, vals[:int(off[-1])]
+
+
 def release_stream(stream=None):
     """Free the library's cached workspace and side stream for `stream` (call
     before destroying a stream the library was used on)."""
@@ -501,4 +525,5 @@ def msm_prepared_sharded(prepared: "PreparedPoints", scalars_local, comm: Comm, 
 __all__ = ["CURVES", "GzkpError", "lib", "msm", "msm_host", "PreparedPoints", "msm_partial", "combine_partials",
            "fixed_base_mul", "field_op", "ec_op", "Comm", "msm_sharded", "msm_prepared_sharded", "shard_range", "set_config",
            "window_bits", "workspace_bytes", "set_profiling", "profile_read", "field_limbs", "scalar_limbs", "to_device",
-           "to_numpy", "ntt", "ntt_max_log", "ntt_last_launches", "scalar_field_op", "release_stream"]
+           "to_numpy", "ntt", "ntt_max_log", "ntt_last_launches", "scalar_field_op", "release_stream",
+           "debug_buckets"]

@@ -162,6 +162,26 @@ cudaError_t pool_malloc(void** p, size_t bytes, cudaStream_t s) {
   return pool ? cudaMallocFromPoolAsync(p, bytes, pool, s) : cudaMallocAsync(p, bytes, s);
 }
 
+bool debug_checks_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("GZKP_DEBUG_CHECKS");
+    return e && atoi(e) != 0;
+  }();
+  return on;
+}
+
+gzkp_status debug_validate(const CurveImpl* c, const void* pts, const void* sc, size_t n, cudaStream_t s) {
+  if (!debug_checks_enabled() || !n) return GZKP_SUCCESS;
+  uint32_t flags = 0;
+  if (gzkp_status st = c->validate(pts, sc, n, &flags, s)) return st;
+  if (!flags) return GZKP_SUCCESS;
+  std::string m = "GZKP_DEBUG_CHECKS:";
+  if (flags & 1) m += " a coordinate is >= p;";
+  if (flags & 2) m += " a point is not on the curve;";
+  if (flags & 4) m += " a scalar is >= 2^b;";
+  return set_error(GZKP_ERROR_INVALID_VALUE, m);
+}
+
 static bool aligned16(const void* p) { return ((uintptr_t)p & 15u) == 0; }
 
 // Per-stream library state, keyed by (device, stream handle, thread): calls
@@ -360,6 +380,7 @@ gzkp_status gzkp_msm_ex(int curve, const void* points_affine, const void* scalar
   const CurveImpl* c = impl_for(curve);
   if (gzkp_status st = check_args(c, points_affine, scalars, n, out)) return st;
   init_pool_once();
+  if (gzkp_status st = debug_validate(c, points_affine, scalars, n, (cudaStream_t)stream)) return st;
   MsmCall call;
   call.points = points_affine;
   call.scalars = scalars;
@@ -381,6 +402,7 @@ gzkp_status gzkp_msm_partial(int curve, const void* points_affine, const void* s
   const CurveImpl* c = impl_for(curve);
   if (gzkp_status st = check_args(c, points_affine, scalars, n, partial_xyzz)) return st;
   init_pool_once();
+  if (gzkp_status st = debug_validate(c, points_affine, scalars, n, (cudaStream_t)stream)) return st;
   MsmCall call;
   call.points = points_affine;
   call.scalars = scalars;
@@ -435,6 +457,10 @@ gzkp_status gzkp_msm_host(int curve, const void* points_host, const void* scalar
   if (!st && (e = cudaEventRecord(ev_points, ss)) != cudaSuccess) st = cuda_status(e, "event");
   if (!st && n && (e = cudaMemcpyAsync(ds, scalars_host, sb, cudaMemcpyHostToDevice, s)) != cudaSuccess)
     st = cuda_status(e, "H2D scalars");
+  if (!st && debug_checks_enabled() && n) {   // staged canonical copies (debug only: synchronises)
+    if ((e = cudaStreamSynchronize(ss)) != cudaSuccess) st = cuda_status(e, "sync");
+    if (!st) st = debug_validate(c, dstage, ds, n, s);
+  }
   if (!st) {
     MsmCall call;
     call.points = dp;
@@ -464,6 +490,7 @@ gzkp_status gzkp_points_prepare_ex(int curve, const void* points_affine, size_t 
   if (weighted != 1 && (window_bits == 1 || window_bits > 16))
     return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..16 for unweighted points");
   if (weighted == 1 && window_bits == 1) return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..22");
+  if (gzkp_status st = debug_validate(c, points_affine, nullptr, n, (cudaStream_t)stream)) return st;
   Prepared* h = new (std::nothrow) Prepared{curve, n, nullptr, false, 0, 1, 0};
   if (!h) return set_error(GZKP_ERROR_OUT_OF_MEMORY, "handle");
   const size_t pt_bytes = 2 * (size_t)c->limbs * 4;
@@ -517,6 +544,7 @@ static gzkp_status msm_prepared_impl(const void* handle, const void* scalars, si
   const CurveImpl* c = impl_for(h->curve);
   if (gzkp_status st = check_args(c, h->pts, scalars, n, out_affine ? out_affine : out_partial)) return st;
   init_pool_once();
+  if (gzkp_status st = debug_validate(c, nullptr, scalars, n, (cudaStream_t)stream)) return st;
   MsmCall call;
   call.points = h->pts;
   call.prepared = true;
@@ -713,6 +741,17 @@ gzkp_status gzkp_msm_prepared_sharded(const void* handle, const void* scalars, s
   if (gzkp_status st = nccl_status(nccl().AllGather(cm->partial, cm->gathered, pb, ncclUint8_, cm->comm, s), "ncclAllGather"))
     return st;
   return c->combine(cm->gathered, cm->world, out, s);
+}
+
+gzkp_status gzkp_debug_buckets(int curve, const void* scalars, size_t n, int window_bits, uint32_t* offsets_host,
+                               size_t offsets_cap, uint32_t* vals_host, size_t vals_cap, gzkp_stream stream) {
+  const CurveImpl* c = impl_for(curve);
+  if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
+  if (window_bits < 2 || window_bits > 16 || !offsets_host || (n && (!scalars || !vals_host)) || !aligned16(scalars))
+    return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
+  init_pool_once();
+  return c->debug_buckets(scalars, n, window_bits, offsets_host, offsets_cap, vals_host, vals_cap,
+                          (cudaStream_t)stream);
 }
 
 gzkp_status gzkp_release_stream(gzkp_stream stream) { return release_stream((cudaStream_t)stream); }

@@ -53,7 +53,16 @@ struct CurveImpl {
   gzkp_status (*ec_op)(int op, const void* P, const void* Q, void* out, size_t n, cudaStream_t s);
   gzkp_status (*precompute)(const void* in, size_t n, int c, void* table, int* c_out, int* w_out, cudaStream_t s);
   int (*table_windows)(size_t n, int c);
+  // GZKP_DEBUG_CHECKS: points (canonical, may be null) / scalars (may be null)
+  // -> flags (bit 0 coordinate >= p, 1 off curve, 2 scalar >= 2^b); synchronises
+  gzkp_status (*validate)(const void* pts, const void* sc, size_t n, uint32_t* flags_host, cudaStream_t s);
+  gzkp_status (*debug_buckets)(const void* sc, size_t n, int c, uint32_t* off_host, size_t off_cap,
+                               uint32_t* vals_host, size_t vals_cap, cudaStream_t s);
 };
+// GZKP_DEBUG_CHECKS=1 in the environment (read once)
+bool debug_checks_enabled();
+// validates when debug checks are on: GZKP_ERROR_INVALID_VALUE on bad inputs
+gzkp_status debug_validate(const CurveImpl* c, const void* pts, const void* sc, size_t n, cudaStream_t s);
 
 const CurveImpl* impl_bn254();
 const CurveImpl* impl_bls12_381();

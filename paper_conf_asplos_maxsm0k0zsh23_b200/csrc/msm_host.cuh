@@ -316,22 +316,13 @@ struct Impl {
     return run(call, p, ws);
   }
 
-  static gzkp_status run(const MsmCall& call, const Plan& p, char* ws) {
+  // a2 + a3: signed-window digits of every (point, window), bucket
+  // histogram, exclusive scan -> offsets[0..M] (offsets[M] = E), and the
+  // scatter of (point index | sign) into bucket order -> vals[0..E).
+  static gzkp_status sort_stage(const MsmCall& call, const Plan& p, char* ws, int* launches) {
     cudaStream_t s = call.stream;
     const size_t n = call.n;
     auto U = [&](size_t off) { return (uint32_t*)(ws + off); };
-    ProfileRecord* prof = profile_begin(s);
-    cudaEvent_t ev_begin = profile_event(prof, s);
-    int launches = 0;
-    const int sms = device_sm_count();
-
-    // a1: points -> Montgomery (skipped for prepared handles)
-    const uint32_t* pts = (const uint32_t*)call.points;
-    if (!call.prepared) {
-      if (gzkp_status st = to_mont_sc(call.points, U(p.o_pts), n, call.scalars, s)) return st;
-      pts = U(p.o_pts);
-      ++launches;
-    }
     // a2: digits + histogram
     GZ_CHECK(cudaMemsetAsync(U(p.o_counts), 0, (size_t)p.M * 4, s));
     GZ_CHECK(cudaMemsetAsync(U(p.o_hot), 0, ((size_t)p.M + 31) / 32 * 4, s));
@@ -352,7 +343,57 @@ struct Impl {
     k_scatter<<<(unsigned)((uint64_t)bpw_s * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw_s, key_stride,
                                                                          p.val_stride, U(p.o_hot), U(p.o_cursor), U(p.o_vals));
     GZ_CHECK(cudaGetLastError());
-    launches += 5;
+    *launches += 5;
+    return GZKP_SUCCESS;
+  }
+
+  // Test hook (gzkp_debug_buckets): the sort stage alone for window bits c;
+  // copies offsets (M + 1 words) and vals (E words) to the host.
+  static gzkp_status debug_buckets(const void* sc, size_t n, int c, uint32_t* off_host, size_t off_cap,
+                                   uint32_t* vals_host, size_t vals_cap, cudaStream_t s) {
+    const Plan p = plan(n, true, false, c);
+    if (off_cap < (size_t)p.M + 1) return set_error(GZKP_ERROR_INVALID_VALUE, "offsets buffer too small");
+    void* ws = nullptr;
+    if (gzkp_status st = stream_workspace(s, p.total, &ws)) return st;
+    MsmCall call;
+    call.scalars = sc;
+    call.n = n;
+    call.prepared = true;
+    call.stream = s;
+    int launches = 0;
+    if (n)
+      if (gzkp_status st = sort_stage(call, p, (char*)ws, &launches)) return st;
+    GZ_CHECK(cudaMemcpyAsync(off_host, (char*)ws + p.o_offsets, ((size_t)p.M + 1) * 4, cudaMemcpyDeviceToHost, s));
+    GZ_CHECK(cudaStreamSynchronize(s));
+    if (!n) {
+      for (size_t k = 0; k <= p.M; ++k) off_host[k] = 0;
+      return GZKP_SUCCESS;
+    }
+    const size_t E = off_host[p.M];
+    if (vals_cap < E) return set_error(GZKP_ERROR_INVALID_VALUE, "vals buffer too small");
+    GZ_CHECK(cudaMemcpyAsync(vals_host, (char*)ws + p.o_vals, E * 4, cudaMemcpyDeviceToHost, s));
+    GZ_CHECK(cudaStreamSynchronize(s));
+    return GZKP_SUCCESS;
+  }
+
+  static gzkp_status run(const MsmCall& call, const Plan& p, char* ws) {
+    cudaStream_t s = call.stream;
+    const size_t n = call.n;
+    auto U = [&](size_t off) { return (uint32_t*)(ws + off); };
+    ProfileRecord* prof = profile_begin(s);
+    cudaEvent_t ev_begin = profile_event(prof, s);
+    int launches = 0;
+    const int sms = device_sm_count();
+
+    // a1: points -> Montgomery (skipped for prepared handles)
+    const uint32_t* pts = (const uint32_t*)call.points;
+    if (!call.prepared) {
+      if (gzkp_status st = to_mont_sc(call.points, U(p.o_pts), n, call.scalars, s)) return st;
+      pts = U(p.o_pts);
+      ++launches;
+    }
+    // a2 + a3: signed digits, bucket histogram, offsets, sort by bucket
+    if (gzkp_status st = sort_stage(call, p, ws, &launches)) return st;
     cudaEvent_t ev_sorted = profile_event(prof, s);
     profile_interval(prof, 0, ev_begin, ev_sorted);
 
@@ -569,11 +610,27 @@ struct Impl {
     return GZKP_SUCCESS;
   }
 
+  static gzkp_status validate(const void* pts, const void* sc, size_t n, uint32_t* flags_host, cudaStream_t s) {
+    *flags_host = 0;
+    if (!n) return GZKP_SUCCESS;
+    uint32_t* f = nullptr;
+    GZ_CHECK(pool_malloc((void**)&f, 4, s));
+    GZ_CHECK(cudaMemsetAsync(f, 0, 4, s));
+    const int threads = 128;
+    const int grid = (int)std::min<size_t>((n + threads - 1) / threads, (size_t)device_sm_count() * 16);
+    k_validate<C><<<grid, threads, 0, s>>>((const uint32_t*)pts, (const uint32_t*)sc, n, f);
+    GZ_CHECK(cudaGetLastError());
+    GZ_CHECK(cudaMemcpyAsync(flags_host, f, 4, cudaMemcpyDeviceToHost, s));
+    GZ_CHECK(cudaFreeAsync(f, s));
+    GZ_CHECK(cudaStreamSynchronize(s));
+    return GZKP_SUCCESS;
+  }
+
   static const CurveImpl* get() {
     static const CurveImpl impl = {C::ID, C::N, C::NS, C::SCALAR_BITS,
                                    &Impl::window_bits, &Impl::workspace_bytes, &Impl::msm, &Impl::to_mont,
                                    &Impl::combine, &Impl::fixed_base, &Impl::field_op, &Impl::ec_op,
-                                   &Impl::precompute, &Impl::table_windows};
+                                   &Impl::precompute, &Impl::table_windows, &Impl::validate, &Impl::debug_buckets};
     return &impl;
   }
 };

@@ -892,6 +892,67 @@ __global__ void __launch_bounds__(128) k_precompute_step(const uint32_t* __restr
   }
 }
 
+// ------------------------------------- input validation (GZKP_DEBUG_CHECKS=1)
+// Off the hot path.  flags |= 1: a coordinate >= p; 2: a point off the curve
+// y^2 = x^3 + a x + b; 4: a scalar >= 2^b.  b is not a product
+// constant: it is recovered from the generator, b = G_y^2 - G_x^3 - a G_x.
+// pts / sc may be null (validate only the other).  (0, 0) is the identity.
+template <class C>
+__global__ void __launch_bounds__(128) k_validate(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ sc,
+                                                  size_t n, uint32_t* __restrict__ flags) {
+  using Fp = Field<C>;
+  using EC_ = EC<C>;
+  constexpr int N = C::N;
+  uint32_t f = 0;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x) {
+    if (sc) {
+      const uint32_t* k = sc + i * C::NS;
+#pragma unroll 1
+      for (int w = C::SCALAR_BITS / 32; w < C::NS; ++w) {
+        const int lo = C::SCALAR_BITS - 32 * w;           // bits >= lo of word w must be 0
+        const uint32_t mask = lo <= 0 ? 0xffffffffu : (lo >= 32 ? 0u : ~((1u << lo) - 1u));
+        if (k[w] & mask) f |= 4u;
+      }
+    }
+    if (!pts) continue;
+    uint32_t x[N], y[N], xm[N], ym[N], t[N];
+    EC_::ld(x, pts + i * 2 * N);
+    EC_::ld(y, pts + i * 2 * N + N);
+    if (Fp::is_zero(x) && Fp::is_zero(y)) continue;
+    Fp::to_mont(xm, x);
+    Fp::to_mont(ym, y);
+    Fp::from_mont(t, xm);
+    bool canon = Fp::eq(t, x);
+    Fp::from_mont(t, ym);
+    canon = canon && Fp::eq(t, y);
+    if (!canon) { f |= 1u; continue; }
+    // f(X, Y) = Y^2 - X^3 - a X, equal to b for every point on the curve
+    auto rhs_gap = [](uint32_t r[N], const uint32_t X[N], const uint32_t Y[N]) {
+      uint32_t u[N], v[N];
+      Fp::sqr(r, Y);
+      Fp::sqr(u, X);
+      Fp::mul(u, u, X);
+      Fp::sub(r, r, u);
+      if constexpr (!C::A_ZERO) {
+        uint32_t a[N];
+#pragma unroll
+        for (int q = 0; q < N; ++q) a[q] = C::A_MONT(q);
+        Fp::mul(v, a, X);
+        Fp::sub(r, r, v);
+      }
+    };
+    uint32_t gx[N], gy[N], bg[N], bp[N];
+#pragma unroll
+    for (int q = 0; q < N; ++q) { gx[q] = C::GX(q); gy[q] = C::GY(q); }
+    Fp::to_mont(gx, gx);
+    Fp::to_mont(gy, gy);
+    rhs_gap(bg, gx, gy);
+    rhs_gap(bp, xm, ym);
+    if (!Fp::eq(bg, bp)) f |= 2u;
+  }
+  if (f) atomicOr(flags, f);
+}
+
 // ---------------------------------------- fixed-base generator (bench inputs)
 template <class C>
 __global__ void __launch_bounds__(128) k_fixed_base(const uint32_t* __restrict__ sc, size_t n,

@@ -189,7 +189,9 @@ def test_g2_fixed_base_vs_oracle(name):
     assert np.array_equal(got, want)
 
 
-@pytest.mark.parametrize("name,logn", [("bn254_g2", 18), ("bls12_381_g2", 17)])
+@pytest.mark.parametrize("name,logn", [("bn254_g2", 18), ("bls12_381_g2", 17),
+                                       # the benched G2 workloads (bench.py *_g2_2p20, planner c = 16)
+                                       ("bn254_g2", 20), ("bls12_381_g2", 20)])
 def test_g2_large_closed_form(name, logn):
     """Larger n: device-generated points a_i G2 (a 16-point sample re-derived by
     the oracle), MSM checked against the oracle's closed form
@@ -204,7 +206,12 @@ def test_g2_large_closed_form(name, logn):
     sample = np.random.Generator(np.random.PCG64(1)).choice(n, 16, replace=False)
     assert np.array_equal(host(P)[sample], oracle.points_from_dlogs(c, d[sample]))
     want = oracle.closed_form(c, k, d)
+    gz.set_profiling(True)
+    gz.profile_read(reset=True)
     assert np.array_equal(host(gz.msm(name, P, dev(k))), want)
+    prof = gz.profile_read(reset=True)
+    gz.set_profiling(False)
+    assert prof["c"] == gz.window_bits(name, n)
     h = gz.PreparedPoints(name, P, weighted=True)
     assert np.array_equal(host(h.msm(dev(k))), want)
     h.release()

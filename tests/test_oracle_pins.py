@@ -297,6 +297,25 @@ def test_dot_mod_exact():
     K = np.array([ref.int_to_limbs(x, 8) for x in k], dtype=np.uint32)
     A = np.array([ref.int_to_limbs(x, 8) for x in a], dtype=np.uint32)
     assert oracle.dot_mod(K, A, c.r) == sum(x * y for x, y in zip(k, a)) % c.r
+    # several chunks (the float64 partial products are summed across chunks)
+    assert oracle.dot_mod(K, A, c.r, chunk=7) == sum(x * y for x, y in zip(k, a)) % c.r
+
+
+def test_dot_mod_tiled_and_extreme_limbs():
+    """a_i = dlogs[i mod m] (SURVEY.md §8(d) tiling) and all-ones limbs, where
+    a chunk's float64 sums are largest (every 16-bit half 0xffff)."""
+    rng = random.Random(2)
+    c = curves.MNT4_753
+    n, m = 1000, 37
+    k = [rng.randrange(c.r) for _ in range(n)]
+    a = [rng.randrange(c.r) for _ in range(m)]
+    K = np.array([ref.int_to_limbs(x, 24) for x in k], dtype=np.uint32)
+    A = np.array([ref.int_to_limbs(x, 24) for x in a], dtype=np.uint32)
+    want = sum(k[i] * a[i % m] for i in range(n)) % c.r
+    assert oracle.dot_mod(K, A, c.r) == want
+    assert oracle.dot_mod(K, A, c.r, chunk=64) == want
+    big = np.full((3000, 24), 0xFFFFFFFF, dtype=np.uint32)
+    assert oracle.dot_mod(big, big, c.r) == (3000 * ((1 << 768) - 1) ** 2) % c.r
 
 
 def test_msm_empty_and_zero():
