@@ -510,6 +510,178 @@ struct F {
     }
     if (is_one_int(u)) copy(r, x1); else copy(r, x2);
   }
+  // ---- constant-time inverse by the optimised binary GCD (Pornin, "Optimized
+  // Binary GCD for Modular Inversion", 2020; tools/emulate_bingcd.py is the
+  // bit-exact model): r = x^-1 mod p for a canonical x (x = 0 gives 0).
+  // T = ceil((2 bits(p) - 1) / 31) outer iterations; each runs 31 divsteps on
+  // 64-bit approximations of (a, b) (31 low + 33 top bits), then applies the
+  // accumulated 2x2 matrix (|f|, |g| <= 2^31) to the full values and, with a
+  // Montgomery division by 2^31, to the Bezout coefficients (u, v), keeping
+  // a = u x and b = v x (mod p) exact.  No data-dependent branch: every lane
+  // of a warp runs the same instruction stream, so a warp inverts 32 values
+  // at the cost of one (the batch-affine accumulation relies on this).
+  static constexpr int BG_OUTER = (2 * C::P_BITS - 1 + 30) / 31;
+  static constexpr int BG_L = N + 2;          // signed working width (limbs)
+
+  // r = |m| * a  (N + 1 limbs) for a u32 magnitude
+  GZ_DEV static void mul_small(uint32_t r[N + 1], const uint32_t a[N], uint32_t m) {
+    r[0] = a[0] * m;
+    uint32_t t = mul_hi(a[0], m);
+#pragma unroll
+    for (int i = 1; i < N; ++i) {
+      MAD_LO_CC(r[i], a[i], m, t);
+      MADC_HI(t, a[i], m, 0u);
+    }
+    r[N] = t;
+  }
+  // z = a f + b g, signed, BG_L limbs two's complement (|f|, |g| <= 2^31)
+  GZ_DEV static void lincomb(uint32_t z[BG_L], const uint32_t a[N], int64_t f, const uint32_t b[N], int64_t g) {
+    uint32_t x[N + 1], y[N + 1];
+    const uint32_t fm = (uint32_t)(f < 0 ? -f : f), gm = (uint32_t)(g < 0 ? -g : g);
+    const uint32_t fs = f < 0 ? 0xffffffffu : 0u, gs = g < 0 ? 0xffffffffu : 0u;
+    mul_small(x, a, fm);
+    mul_small(y, b, gm);
+    // two's complement negation of a magnitude: (x ^ s) + (s & 1)
+    uint32_t xs[BG_L], ys[BG_L];
+#pragma unroll
+    for (int i = 0; i <= N; ++i) { xs[i] = x[i] ^ fs; ys[i] = y[i] ^ gs; }
+    xs[N + 1] = fs;
+    ys[N + 1] = gs;
+    ADD_CC(z[0], xs[0], ys[0]);
+#pragma unroll
+    for (int i = 1; i < BG_L; ++i) ADDC_CC(z[i], xs[i], ys[i]);
+    // + (fs & 1) + (gs & 1): add the two's-complement corrections
+    uint32_t corr = (fs & 1u) + (gs & 1u);
+    ADD_CC(z[0], z[0], corr);
+#pragma unroll
+    for (int i = 1; i < BG_L - 1; ++i) ADDC_CC(z[i], z[i], 0u);
+    ADDC(z[BG_L - 1], z[BG_L - 1], 0u);
+  }
+  // arithmetic shift right by 31 of a BG_L-limb signed value, to N + 1 limbs
+  GZ_DEV static void sar31(uint32_t r[N + 1], const uint32_t z[BG_L]) {
+#pragma unroll
+    for (int i = 0; i <= N; ++i) r[i] = __funnelshift_r(z[i], z[i + 1], 31);
+  }
+  GZ_DEV static void neg_n1(uint32_t r[N + 1], uint32_t s) {   // r = s ? -r : r
+#pragma unroll
+    for (int i = 0; i <= N; ++i) r[i] ^= s;
+    ADD_CC(r[0], r[0], s & 1u);
+#pragma unroll
+    for (int i = 1; i < N; ++i) ADDC_CC(r[i], r[i], 0u);
+    ADDC(r[N], r[N], 0u);
+  }
+  // r (N + 1 limbs, signed, |r| < 3p)  ->  canonical in [0, p)
+  GZ_DEV static void normalize_signed(uint32_t out[N], uint32_t r[N + 1]) {
+#pragma unroll
+    for (int k = 0; k < 3; ++k) {          // add p while negative
+      const uint32_t s = (uint32_t)((int32_t)r[N] >> 31);
+      ADD_CC(r[0], r[0], C::P(0) & s);
+#pragma unroll
+      for (int i = 1; i < N; ++i) ADDC_CC(r[i], r[i], C::P(i) & s);
+      ADDC(r[N], r[N], 0u);
+    }
+#pragma unroll
+    for (int k = 0; k < 2; ++k) {          // subtract p while >= p
+      uint32_t t[N + 1];
+      SUB_CC(t[0], r[0], C::P(0));
+#pragma unroll
+      for (int i = 1; i < N; ++i) SUBC_CC(t[i], r[i], C::P(i));
+      SUBC(t[N], r[N], 0u);
+      const uint32_t keep = (uint32_t)((int32_t)t[N] >> 31);   // all ones: r < p
+#pragma unroll
+      for (int i = 0; i <= N; ++i) r[i] = keep ? r[i] : t[i];
+    }
+#pragma unroll
+    for (int i = 0; i < N; ++i) out[i] = r[i];
+  }
+  // (u f + v g) / 2^31 mod p, u, v canonical
+  GZ_DEV static void bezout_update(uint32_t out[N], const uint32_t u[N], int64_t f, const uint32_t v[N], int64_t g) {
+    uint32_t z[BG_L], tp[N + 1];
+    lincomb(z, u, f, v, g);
+    const uint32_t t = (z[0] * C::N0) & 0x7fffffffu;     // z + t p = 0 mod 2^31
+    uint32_t pp[N];
+#pragma unroll
+    for (int i = 0; i < N; ++i) pp[i] = C::P(i);
+    mul_small(tp, pp, t);
+    ADD_CC(z[0], z[0], tp[0]);
+#pragma unroll
+    for (int i = 1; i <= N; ++i) ADDC_CC(z[i], z[i], tp[i]);
+    ADDC(z[N + 1], z[N + 1], 0u);
+    uint32_t r[N + 1];
+    sar31(r, z);
+    normalize_signed(out, r);
+  }
+  __device__ __noinline__ static void inv_bingcd(uint32_t* r, const uint32_t* x) {
+    uint32_t a[N], b[N], u[N], v[N];
+#pragma unroll
+    for (int i = 0; i < N; ++i) { a[i] = x[i]; b[i] = C::P(i); u[i] = 0; v[i] = 0; }
+    u[0] = 1;
+#pragma unroll 1
+    for (int it = 0; it < BG_OUTER; ++it) {
+      // n = max(len(a), len(b), 64); window [n - 33, n) of a and b
+      uint32_t top = 0;
+      int idx = 0;
+#pragma unroll
+      for (int i = 0; i < N; ++i) {
+        const uint32_t o = a[i] | b[i];
+        top = o ? o : top;
+        idx = o ? i : idx;
+      }
+      int len = top ? 32 * idx + 32 - __clz(top) : 0;
+      len = len < 64 ? 64 : len;
+      const int s = len - 33, w = s >> 5, sh = s & 31;
+      uint32_t al = 0, am = 0, ah = 0, bl = 0, bm = 0, bh = 0;
+#pragma unroll
+      for (int i = 0; i < N; ++i) {
+        al = i == w ? a[i] : al;     am = i == w + 1 ? a[i] : am;     ah = i == w + 2 ? a[i] : ah;
+        bl = i == w ? b[i] : bl;     bm = i == w + 1 ? b[i] : bm;     bh = i == w + 2 ? b[i] : bh;
+      }
+      const uint32_t at = __funnelshift_r(al, am, sh), atb = __funnelshift_r(am, ah, sh) & 1u;
+      const uint32_t bt = __funnelshift_r(bl, bm, sh), btb = __funnelshift_r(bm, bh, sh) & 1u;
+      uint64_t xa = ((uint64_t)((atb << 31) | (at >> 1)) << 32) | ((at << 31) | (a[0] & 0x7fffffffu));
+      uint64_t xb = ((uint64_t)((btb << 31) | (bt >> 1)) << 32) | ((bt << 31) | (b[0] & 0x7fffffffu));
+      int64_t f0 = 1, g0 = 0, f1 = 0, g1 = 1;
+#pragma unroll 1
+      for (int j = 0; j < 31; ++j) {
+        const uint64_t mo = 0ull - (xa & 1ull);                  // a odd
+        const uint64_t ms = mo & (0ull - (uint64_t)(xa < xb));  // odd and a < b: swap
+        const uint64_t tx = (xa ^ xb) & ms;
+        xa ^= tx;
+        xb ^= tx;
+        const int64_t tf = (f0 ^ f1) & (int64_t)ms, tg = (g0 ^ g1) & (int64_t)ms;
+        f0 ^= tf; f1 ^= tf;
+        g0 ^= tg; g1 ^= tg;
+        xa -= xb & mo;
+        f0 -= f1 & (int64_t)mo;
+        g0 -= g1 & (int64_t)mo;
+        xa >>= 1;
+        f1 += f1;
+        g1 += g1;
+      }
+      // (a, b) <- ((a f0 + b g0) / 2^31, (a f1 + b g1) / 2^31), made non-negative
+      uint32_t za[BG_L], zb[BG_L], ra[N + 1], rb[N + 1];
+      lincomb(za, a, f0, b, g0);
+      lincomb(zb, a, f1, b, g1);
+      sar31(ra, za);
+      sar31(rb, zb);
+      const uint32_t sa = (uint32_t)((int32_t)za[BG_L - 1] >> 31), sb = (uint32_t)((int32_t)zb[BG_L - 1] >> 31);
+      neg_n1(ra, sa);
+      neg_n1(rb, sb);
+      f0 = sa ? -f0 : f0;  g0 = sa ? -g0 : g0;
+      f1 = sb ? -f1 : f1;  g1 = sb ? -g1 : g1;
+#pragma unroll
+      for (int i = 0; i < N; ++i) { a[i] = ra[i]; b[i] = rb[i]; }
+      uint32_t nu[N], nv[N];
+      bezout_update(nu, u, f0, v, g0);
+      bezout_update(nv, u, f1, v, g1);
+#pragma unroll
+      for (int i = 0; i < N; ++i) { u[i] = nu[i]; v[i] = nv[i]; }
+    }
+    // b = gcd(x, p) = 1 for x != 0: v = x^-1; x = 0 leaves b = p, v = 0
+#pragma unroll
+    for (int i = 0; i < N; ++i) r[i] = v[i];
+  }
+
   // Montgomery-domain inverse: (aR)^-1 R = from/to conversions around EEA
   GZ_DEV static void inv(uint32_t r[N], const uint32_t a[N]) {
     uint32_t c[N], ic[N];

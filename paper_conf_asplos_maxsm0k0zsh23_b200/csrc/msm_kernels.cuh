@@ -1002,6 +1002,9 @@ __global__ void k_field_op(int op, const uint32_t* __restrict__ a, const uint32_
       case 1: Fp::add(r, x, y); break;
       case 2: Fp::sub(r, x, y); break;
       case 3: Fp::inv_canonical(r, x); break;
+      case 7:   // constant-time binary-GCD inverse (canonical in / out), F_p curves
+        if constexpr (std::is_same<Fp, F<C>>::value) Fp::inv_bingcd(r, x); else Fp::inv_canonical(r, x);
+        break;
       case 5: Fp::to_mont(x, x); Fp::sqr(r, x); Fp::from_mont(r, r); break;
       case 6:   // FP64 (DFP) Montgomery product where available, else the IMAD one
         Fp::to_mont(x, x); Fp::to_mont(y, y);

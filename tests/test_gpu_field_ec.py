@@ -56,8 +56,30 @@ def test_field_ops(c):
         assert limbs_int(rt[i]) == a[i], i
     nz = [x for x in a if x][:3000]
     inv = host(gz.field_op(c.name, 3, dev(int_limbs(nz, L)), dev(int_limbs(nz, L))))
+    bg = host(gz.field_op(c.name, 7, dev(int_limbs(nz, L)), dev(int_limbs(nz, L))))   # binary-GCD inverse
     for i, x in enumerate(nz):
         assert limbs_int(inv[i]) == pow(x, -1, c.p), (i, x)
+        assert limbs_int(bg[i]) == pow(x, -1, c.p), ("bingcd", i, x)
+    assert not host(gz.field_op(c.name, 7, dev(int_limbs([0], L)), dev(int_limbs([0], L)))).any()
+
+
+@pytest.mark.parametrize("c", [curves.BN254, curves.BLS12_381, curves.MNT4_753], ids=lambda c: c.name)
+def test_bingcd_inverse_stress(c):
+    """The constant-time binary-GCD inverse (Pornin's bound of
+    ceil((2 len p - 1) / 31) outer iterations) on many random values and on
+    values with long runs of zero / one bits: x x^-1 = 1 (mod p)."""
+    gz = require_cuda()
+    rng = random.Random(99 + c.cid)
+    L = c.limbs
+    n = 1 << (17 if L <= 12 else 14)
+    xs = [rng.randrange(1, c.p) for _ in range(n)]
+    xs += [(1 << k) % c.p for k in range(c.p.bit_length())]
+    xs += [((1 << k) - 1) % c.p or 1 for k in range(1, c.p.bit_length())]
+    xs += [c.p - (1 << k) for k in range(c.p.bit_length() - 1)]
+    X = dev(int_limbs(xs, L))
+    got = host(gz.field_op(c.name, 7, X, X))
+    for i, x in enumerate(xs):
+        assert limbs_int(got[i]) * x % c.p == 1, (i, x)
 
 
 def _points(c, k, seed):
