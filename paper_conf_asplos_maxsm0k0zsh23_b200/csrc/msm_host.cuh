@@ -31,6 +31,11 @@ struct Plan {
   uint32_t val_stride = 0;     // table stride of the weighted points (consolidated)
   uint32_t M = 0;        // Wb * B bucket keys
   int S = 64;            // entries per accumulation chunk
+  // batch-affine levels (affine.cuh): level arrays A (odd levels) / B (even),
+  // their offsets, the thread-distribution offsets, per-thread prefix scratch
+  int aff_levels = 0;
+  uint32_t aff_ctas = 0;
+  size_t o_aoff = 0, o_aoffA = 0, o_aoffB = 0, o_lvlA = 0, o_lvlB = 0, o_ascr = 0;
   int seg = 16;          // buckets per reduction segment
   int heavy_levels = 0;  // depth of the heavy-bucket tree (max over groups)
   size_t n = 0;
@@ -157,6 +162,27 @@ struct Impl {
     return best;
   }
 
+  // Batch-affine levels before the XYZZ hot loop (affine.cuh): enough halvings
+  // that an average bucket (E / M entries) is finished, at most 8 (a heavier
+  // bucket -- the sparse witness's bucket 1 -- is left to the XYZZ chunks and
+  // the heavy-bucket tree).  GZKP_AFFINE_LEVELS overrides (0 = XYZZ only).
+  static int affine_levels(const Plan& p) {
+    if constexpr (!AffineCfg<C>::ON) {
+      return 0;
+    } else {
+      static const int env = [] {
+        const char* e = getenv("GZKP_AFFINE_LEVELS");
+        return e ? atoi(e) : -1;
+      }();
+      if (env >= 0) return std::min(env, 16);
+      if (!AffineCfg<C>::DEFAULT_ON) return 0;
+      const double avg = (double)p.E_max / (double)std::max<uint32_t>(p.M, 1);
+      int L = 0;
+      while (L < 8 && std::ldexp(1.0, L) < avg) ++L;
+      return L;
+    }
+  }
+
   static Plan plan(size_t n, bool prepared, bool consolidated = false, int c_forced = 0, size_t table_n = 0) {
     Plan p;
     p.n = n;
@@ -265,6 +291,20 @@ struct Impl {
     p.o_mid = take((size_t)mid_elems * 4 * N * 4);
     p.o_terms = take((size_t)terms_elems * 4 * N * 4);
     p.o_win = take((size_t)p.Wb * 4 * N * 4);
+    // batch-affine levels: E_{l+1} <= E_l / 2 + min(M, E_l / 3) / 2 (a bucket
+    // of c >= 3 entries keeps ceil(c / 2) <= (c + 1) / 2; c <= 2 finishes)
+    p.aff_levels = affine_levels(p);
+    if (p.aff_levels > 0) {
+      auto next_cap = [&](uint64_t cap) { return cap / 2 + std::min<uint64_t>(p.M, cap / 3) / 2 + 1; };
+      const uint64_t cap1 = next_cap(p.E_max), cap2 = next_cap(cap1);
+      p.aff_ctas = (uint32_t)device_sm_count() * AffineCfg<C>::MINB;
+      p.o_aoff = take(((size_t)p.M + 1) * 4);
+      p.o_aoffA = take(((size_t)p.M + 1) * 4);
+      p.o_aoffB = take(((size_t)p.M + 1) * 4);
+      p.o_lvlA = take(cap1 * 2 * N * 4);
+      p.o_lvlB = take(p.aff_levels > 1 ? cap2 * 2 * N * 4 : 4);
+      p.o_ascr = take((size_t)p.aff_ctas * AffineCfg<C>::THREADS * AffineCfg<C>::BL * N * 4);
+    }
     p.total = o;
     return p;
   }
@@ -376,6 +416,52 @@ struct Impl {
     return GZKP_SUCCESS;
   }
 
+  // exclusive scan of in[0..count) -> out[0..count), out[count] = total
+  static gzkp_status scan(const uint32_t* in, uint32_t* out, uint32_t count, uint32_t* tiles, cudaStream_t s) {
+    const uint32_t ntiles = (count + SCAN_TILE - 1) / SCAN_TILE;
+    if (ntiles > (uint32_t)SCAN_TILE) return set_error(GZKP_ERROR_INVALID_VALUE, "scan too large");
+    k_scan_tiles<<<ntiles, SCAN_THREADS, 0, s>>>(in, out, count, tiles, nullptr);
+    k_scan_top<<<1, SCAN_THREADS, 0, s>>>(tiles, ntiles, out + count);
+    k_scan_add<<<ntiles, SCAN_THREADS, 0, s>>>(out, nullptr, count, tiles);
+    GZ_CHECK(cudaGetLastError());
+    return GZKP_SUCCESS;
+  }
+
+  // a4, batch-affine levels (affine.cuh): halve every bucket p.aff_levels
+  // times; buckets left with one element are written to the bucket array.
+  // Returns the residual level array and its offsets for the XYZZ hot loop.
+  static gzkp_status affine_stage(const Plan& p, char* ws, const uint32_t* pts, cudaStream_t s,
+                                  const uint32_t** offs_out, const uint32_t** pts_out, int* launches) {
+    auto U = [&](size_t off) { return (uint32_t*)(ws + off); };
+    const uint32_t* off_in = U(p.o_offsets);
+    const uint32_t* in = pts;
+    for (int l = 0; l < p.aff_levels; ++l) {
+      uint32_t* cnt_out = U(p.o_counts);       // dead after the sort
+      uint32_t* cnt_next = U(p.o_cursor);
+      uint32_t* off_out = U(p.o_aoff);
+      uint32_t* off_next = U((l & 1) ? p.o_aoffB : p.o_aoffA);
+      uint32_t* out = U((l & 1) ? p.o_lvlB : p.o_lvlA);
+      k_level_counts<<<(p.M + 255) / 256, 256, 0, s>>>(off_in, p.M, cnt_out, cnt_next);
+      GZ_CHECK(cudaGetLastError());
+      if (gzkp_status st = scan(cnt_out, off_out, p.M, U(p.o_tiles), s)) return st;
+      if (gzkp_status st = scan(cnt_next, off_next, p.M, U(p.o_tiles), s)) return st;
+      const size_t smem = (size_t)AffineCfg<C>::THREADS * AffineIn<C, true>::SLOT_WORDS * 4;
+      if (l == 0)
+        k_affine_level<C, true><<<p.aff_ctas, AffineCfg<C>::THREADS, smem, s>>>(
+            U(p.o_vals), in, off_in, off_out, off_next, p.M, out, U(p.o_buckets), U(p.o_ascr));
+      else
+        k_affine_level<C, false><<<p.aff_ctas, AffineCfg<C>::THREADS, smem, s>>>(
+            nullptr, in, off_in, off_out, off_next, p.M, out, U(p.o_buckets), U(p.o_ascr));
+      GZ_CHECK(cudaGetLastError());
+      *launches += 8;
+      off_in = off_next;
+      in = out;
+    }
+    *offs_out = off_in;
+    *pts_out = in;
+    return GZKP_SUCCESS;
+  }
+
   static gzkp_status run(const MsmCall& call, const Plan& p, char* ws) {
     cudaStream_t s = call.stream;
     const size_t n = call.n;
@@ -437,6 +523,14 @@ struct Impl {
           if constexpr (AccumCfg<C>::DFP)
             GZ_CHECK(cudaFuncSetAttribute(k_accum<C, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                           (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
+          GZ_CHECK(cudaFuncSetAttribute(k_accum<C, false, AccumCfg<C>::MIN_CTAS, true>,
+                                        cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                        (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
+          if constexpr (AffineCfg<C>::ON) {
+            const int asm_ = (int)((size_t)AffineCfg<C>::THREADS * AffineIn<C, true>::SLOT_WORDS * 4);
+            GZ_CHECK(cudaFuncSetAttribute(k_affine_level<C, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, asm_));
+            GZ_CHECK(cudaFuncSetAttribute(k_affine_level<C, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, asm_));
+          }
           GZ_CHECK(cudaFuncSetAttribute(k_reduce_bits<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         (int)((size_t)RB_THREADS * 4 * N * 4)));
           GZ_CHECK(cudaFuncSetAttribute(k_heavy_tree<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -448,6 +542,10 @@ struct Impl {
     // stream while the digits / sort ran; only the accumulation needs them
     if (call.points_ready) GZ_CHECK(cudaStreamWaitEvent(s, call.points_ready, 0));
     cudaEvent_t ev_last_acc = nullptr, ev_merged = nullptr, ev_reduced = nullptr, ev_tailed = nullptr;
+    // bucket layout of the accumulation's input (the residual level array's
+    // after batch-affine levels); the reduction keeps the sorted layout's
+    // offsets for "bucket non-empty"
+    const uint32_t* offs = U(p.o_offsets);
     for (int gi = 0; gi < ngroups; ++gi) {
       const auto& gr = p.groups[gi];
       const Group grp{gr.key_lo, gr.key_hi, (uint32_t)gr.chunk_base};
@@ -456,7 +554,18 @@ struct Impl {
       // a4 (main stream)
       cudaEvent_t a0 = profile_event(prof, s);
       const unsigned acc_grid = (unsigned)((gr.chunks_max + acc_threads - 1) / acc_threads);
-      if constexpr (AccumCfg<C>::DFP) {
+      bool affine = false;
+      if constexpr (AffineCfg<C>::ON) {
+        if (p.aff_levels > 0 && ngroups == 1) {
+          const uint32_t* apts = nullptr;
+          if (gzkp_status st = affine_stage(p, ws, pts, s, &offs, &apts, &launches)) return st;
+          k_accum<C, false, AccumCfg<C>::MIN_CTAS, true><<<acc_grid, acc_threads, acc_smem, s>>>(
+              nullptr, offs, grp, apts, p.S, U(p.o_buckets), U(p.o_spay), mlist, mcnt);
+          affine = true;
+        }
+      }
+      if (affine) {
+      } else if constexpr (AccumCfg<C>::DFP) {
         if (mixed)
           k_accum<C, true><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
                                                                    U(p.o_buckets), U(p.o_spay), mlist, mcnt);
@@ -484,7 +593,7 @@ struct Impl {
       uint4* hlist = (uint4*)U(p.o_hlist) + gr.hbase;
       uint32_t* hjobs = U(p.o_hjobs) + (size_t)std::max(p.heavy_levels, 1) * (gr.hbase + gi);
       const int gm = (int)std::min<uint64_t>((gr.chunks_max + threads - 1) / threads, (uint64_t)sms * 16);
-      k_merge_bucket<C><<<gm, threads, 0, ss>>>(U(p.o_offsets), grp, p.S, mlist, mcnt, U(p.o_spay), U(p.o_buckets),
+      k_merge_bucket<C><<<gm, threads, 0, ss>>>(offs, grp, p.S, mlist, mcnt, U(p.o_spay), U(p.o_buckets),
                                                 heavy, hlist, gr.hmax);
       GZ_CHECK(cudaGetLastError());
       if (gr.heavy_levels > 0) {

@@ -315,7 +315,7 @@ static __global__ void k_scan_tiles(const uint32_t* __restrict__ in, uint32_t* _
   for (int k = 0; k < SCAN_PER_THREAD; ++k) {
     v[k] = (base + k < M) ? in[base + k] : 0u;
     s += v[k];
-    if (v[k] > HOT_COUNT) atomicOr(&hotbits[(base + k) >> 5], 1u << ((base + k) & 31));   // hotbits zeroed by the host
+    if (hotbits && v[k] > HOT_COUNT) atomicOr(&hotbits[(base + k) >> 5], 1u << ((base + k) & 31));   // zeroed by the host
   }
   uint32_t total;
   uint32_t ex = block_exclusive_scan(s, ws, &total);
@@ -355,7 +355,7 @@ static __global__ void k_scan_add(uint32_t* __restrict__ out, uint32_t* __restri
     if (base + k < M) {
       const uint32_t v = out[base + k] + add;
       out[base + k] = v;
-      cursor[base + k] = v;
+      if (cursor) cursor[base + k] = v;
     }
   }
 }
@@ -428,7 +428,10 @@ struct AccumCfg {
 // that merges / reduces / combines the previous group.
 // MINB overrides the register budget (GZKP_ACCUM_MINB=3 selects 3 CTAs / SM,
 // <= 168 registers, for BLS12-381; see msm_host.cuh).
-template <class C, bool MIXED = false, int MINB = AccumCfg<C>::MIN_CTAS>
+// DIRECT: the entries are the points themselves (entry j = point j of `pts`,
+// no index array, no sign): the residual level array of the batch-affine
+// levels (affine.cuh).
+template <class C, bool MIXED = false, int MINB = AccumCfg<C>::MIN_CTAS, bool DIRECT = false>
 __global__ void __launch_bounds__(128, MINB)
     k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off, Group grp,
             const uint32_t* __restrict__ pts, int S, uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay,
@@ -461,14 +464,14 @@ __global__ void __launch_bounds__(128, MINB)
     else EC_::store(spay + (size_t)(open_l ? sidx : sidx + 1) * 4 * N, acc);
   };
 
-  uint32_t v_next = vals[beg];
+  uint32_t v_next = DIRECT ? beg : vals[beg];
   St::fetch(slot, pts, v_next & ~VAL_NEG);
   cp_async_commit();
   for (uint32_t j = beg; j < end; ++j) {
     const uint32_t v = v_next;
     const int buf = (j - beg) & 1;
     if (j + 1 < end) {
-      v_next = vals[j + 1];
+      v_next = DIRECT ? j + 1 : vals[j + 1];
       St::fetch(slot + (buf ^ 1) * St::PT_WORDS, pts, v_next & ~VAL_NEG);
     }
     cp_async_commit();
@@ -1062,3 +1065,5 @@ __global__ void k_ec_op(int op, const uint32_t* __restrict__ P, const uint32_t* 
 }
 
 }  // namespace gzkp
+
+#include "affine.cuh"

@@ -6,6 +6,8 @@ because the switches are read once per process:
 * GZKP_PIPELINE=2      two equal window groups
 * GZKP_ACCUM_THREADS=32  small accumulation CTAs
 * GZKP_WINDOW_BITS / GZKP_SEGMENT  planner overrides
+* GZKP_AFFINE_LEVELS=L  batch-affine tree levels before the XYZZ loop
+                       (affine.cuh experiment; mnt4 and toy curves included)
 """
 
 import os
@@ -27,8 +29,8 @@ from tests.fixtures import oracle_points, oracle_msm_cached
 import paper_conf_asplos_maxsm0k0zsh23_b200 as gz
 ok = True
 for curve, n, dist in (("bls12_381", 1024, "uniform"), ("bls12_381", 1000, "zcash_like"), ("bn254", 1024, "uniform"),
-                       ("toy_a2", 2000, "uniform")):
-    pts, _ = oracle_points(curve, 2048 if curve == "toy_a2" else 1024)
+                       ("toy_a2", 2000, "uniform"), ("toy_a0", 3000, "uniform"), ("mnt4_753", 64, "uniform")):
+    pts, _ = oracle_points(curve, {"toy_a2": 2048, "toy_a0": 4096, "mnt4_753": 64}.get(curve, 1024))
     pts = pts[:n]
     k = synth.scalars(curve, n, 91, dist)
     want = oracle_msm_cached(curve, pts, k)
@@ -42,7 +44,9 @@ print("VARIANT_OK" if ok else "VARIANT_FAIL")
 
 @pytest.mark.parametrize("env", [{"GZKP_DFP": "1"}, {"GZKP_PIPELINE": "1"}, {"GZKP_PIPELINE": "2"}, {"GZKP_ACCUM_THREADS": "32"},
                                  {"GZKP_WINDOW_BITS": "11", "GZKP_SEGMENT": "5"},
-                                 {"GZKP_DFP": "1", "GZKP_PIPELINE": "1", "GZKP_ACCUM_THREADS": "64"}],
+                                 {"GZKP_DFP": "1", "GZKP_PIPELINE": "1", "GZKP_ACCUM_THREADS": "64"},
+                                 {"GZKP_AFFINE_LEVELS": "3"}, {"GZKP_AFFINE_LEVELS": "12"},
+                                 {"GZKP_AFFINE_LEVELS": "2", "GZKP_WINDOW_BITS": "5"}],
                          ids=lambda e: ",".join(f"{k}={v}" for k, v in e.items()))
 def test_variant_parity(env):
     require_cuda()
