@@ -112,17 +112,24 @@ gzkp_status gzkp_msm_host(int curve, const void *points_affine_host, const void 
 
 /* --- prepared points, PAPER.md:194 ("P ... remains unchanged for a specific
  * application", so it is preprocessed once) ------------------------------
- * weighted = 1: GZKP's cross-window consolidation (§4.1,
- *   interval M = 1): the library stores the weighted points 2^(c t) P_i for
- *   every window t (W = ceil((b+1)/c) copies, W*n*2*field_bytes bytes of HBM),
- *   so all windows accumulate into ONE bucket set and the window reduction
- *   disappears.  window_bits = 0 lets the planner choose c, else 2..22; later
- *   MSMs on the handle use that c.
+ * weighted = M >= 1: GZKP's cross-window consolidation with checkpoint
+ *   interval M (§4.1, Algorithm 1): the library stores the
+ *   checkpoints 2^(c M j) P_i for j < ceil(W/M), W = ceil((b+1)/c) (that many
+ *   copies of n*2*field_bytes bytes of HBM).  Window t = M j + r then uses
+ *   checkpoint j and bucket set r, so the W windows accumulate into M bucket
+ *   sets; the remaining weight 2^(c r) is applied once per bucket set to its
+ *   reduced sum (reading R10), not per point as Alg. 1 lines 8-9 do.
+ *   M = 1: the full weighted table, one bucket set, no window combination.
+ *   M >= W: no table beyond the points themselves (the standard pipeline).
+ *   window_bits = 0 lets the planner choose c, else 2..22; later MSMs on the
+ *   handle use that c.
  * weighted = 0: Montgomery-form copy of the points only (standard pipeline);
  *   window_bits 0 (planner per call) or 2..16 (fixed c for every call).
  *   Other values: GZKP_ERROR_INVALID_VALUE.
  * gzkp_points_prepare = _ex(window_bits 0, weighted 1), falling back to
- * weighted 0 if the table does not fit. */
+ * weighted 0 if the table does not fit.  gzkp_prepared_info reports the window
+ * bits, the number of table copies (1 for weighted = 0), the interval M (0 for
+ * unweighted) and the bytes held. */
 gzkp_status gzkp_points_prepare_ex(int curve, const void *points_affine, size_t n, int window_bits,
                                    int weighted, void **handle, gzkp_stream stream);
 gzkp_status gzkp_points_prepare(int curve, const void *points_affine, size_t n, void **handle,
@@ -202,8 +209,12 @@ gzkp_status gzkp_debug_buckets(int curve, const void *scalars, size_t n, int win
 /* Elementwise field ops on canonical inputs (device arrays of n elements):
  * op 0: a*b mod p, 1: a+b, 2: a-b, 3: a^-1 (a != 0), 4: round trip to/from Montgomery,
  * 5: a^2 mod p (the dedicated Montgomery squaring), 6: a*b mod p by the FP64
- * (DFP) Montgomery product where the curve has one (BLS12-381, MNT4-753; NEXT-2),
- * else the IMAD product.  For G2 curves the elements are F_p^2 values c0 || c1. */
+ * (DFP) Montgomery product, which exists for BLS12-381 only (8 x 48-bit limbs;
+ * NEXT-2, measured slower than the IMAD product and off by default); every
+ * other curve, MNT4-753 included, computes op 6 with the IMAD product,
+ * 7: a^-1 mod p by the constant-time binary GCD (the batch-affine inverse;
+ * G2 curves fall back to op 3).  For G2 curves the elements are F_p^2 values
+ * c0 || c1. */
 gzkp_status gzkp_field_op(int curve, int op, const void *a, const void *b, void *out, size_t n,
                           gzkp_stream stream);
 /* Elementwise group ops on canonical affine points (device, n points each):

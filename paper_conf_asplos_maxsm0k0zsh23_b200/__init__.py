@@ -242,9 +242,10 @@ def msm_host(curve, points: np.ndarray, scalars: np.ndarray, out: Optional[np.nd
 class PreparedPoints:
     """Device-resident Montgomery copy of a fixed point vector."""
 
-    def __init__(self, curve, points, stream=None, weighted: Optional[bool] = None, window_bits: int = 0):
+    def __init__(self, curve, points, stream=None, weighted=None, window_bits: int = 0):
         """weighted=None: library default (weighted-point table when it fits);
-        True/False force GZKP's cross-window consolidation on/off."""
+        True/False force GZKP's cross-window consolidation on/off; an int
+        M >= 1 selects Algorithm 1's checkpoint interval M (1 = full table)."""
         self.curve = curve_id(curve)
         self.handle = None
         L = field_limbs(self.curve)
@@ -257,16 +258,23 @@ class PreparedPoints:
                 _check(lib().gzkp_points_prepare(self.curve, P.data_ptr(), self.n, ctypes.byref(h),
                                                  _stream_ptr(stream, P.device)), "gzkp_points_prepare")
             else:
-                _check(lib().gzkp_points_prepare_ex(self.curve, P.data_ptr(), self.n, window_bits,
-                                                    1 if (weighted is None or weighted) else 0, ctypes.byref(h),
-                                                    _stream_ptr(stream, P.device)), "gzkp_points_prepare_ex")
+                if weighted is None or weighted is True:
+                    interval = 1
+                elif weighted is False:
+                    interval = 0
+                else:
+                    interval = int(weighted)
+                _check(lib().gzkp_points_prepare_ex(self.curve, P.data_ptr(), self.n, window_bits, interval,
+                                                    ctypes.byref(h), _stream_ptr(stream, P.device)),
+                       "gzkp_points_prepare_ex")
         self.handle = h
 
     def info(self):
         c, w, wt, b = ctypes.c_int(), ctypes.c_int(), ctypes.c_int(), ctypes.c_size_t()
         _check(lib().gzkp_prepared_info(self.handle, ctypes.byref(c), ctypes.byref(w), ctypes.byref(wt),
                                         ctypes.byref(b)), "gzkp_prepared_info")
-        return {"window_bits": c.value, "windows": w.value, "weighted": bool(wt.value), "bytes": b.value}
+        return {"window_bits": c.value, "windows": w.value, "weighted": bool(wt.value), "interval": wt.value,
+                "bytes": b.value}
 
     def msm(self, scalars, out=None, stream=None):
         torch = _torch()

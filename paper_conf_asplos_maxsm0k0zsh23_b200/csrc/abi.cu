@@ -273,10 +273,11 @@ static gzkp_status release_stream(cudaStream_t s) {
 struct Prepared {
   int curve;
   size_t n;
-  void* pts;          // Montgomery affine: n x 2N u32, or the W x n weighted-point table
-  bool weighted;      // NEXT-1 table 2^(ct) P_i (cross-window consolidation)
-  int c, W;
+  void* pts;          // Montgomery affine: n x 2N u32, or the copies x n checkpoint table
+  bool weighted;      // NEXT-1 checkpoint table 2^(c M j) P_i (cross-window consolidation)
+  int c, W;           // window bits; table copies (weighted) or 1
   size_t bytes;
+  int interval;       // Algorithm 1 checkpoint interval M (weighted only)
 };
 
 // ------------------------------------------------------------- NCCL (dlopen)
@@ -487,21 +488,23 @@ gzkp_status gzkp_points_prepare_ex(int curve, const void* points_affine, size_t 
   if (!handle || (n && !points_affine) || !aligned16(points_affine) || window_bits < 0 || window_bits > 22)
     return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
   // the standard (per-window bucket sets) pipeline plans c <= 16, as gzkp_set_config
-  if (weighted != 1 && (window_bits == 1 || window_bits > 16))
+  if (weighted < 0) return set_error(GZKP_ERROR_INVALID_VALUE, "weighted (checkpoint interval) must be >= 0");
+  if (weighted == 0 && (window_bits == 1 || window_bits > 16))
     return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..16 for unweighted points");
-  if (weighted == 1 && window_bits == 1) return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..22");
+  if (weighted >= 1 && window_bits == 1) return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..22");
   if (gzkp_status st = debug_validate(c, points_affine, nullptr, n, (cudaStream_t)stream)) return st;
-  Prepared* h = new (std::nothrow) Prepared{curve, n, nullptr, false, 0, 1, 0};
+  Prepared* h = new (std::nothrow) Prepared{curve, n, nullptr, false, 0, 1, 0, 1};
   if (!h) return set_error(GZKP_ERROR_OUT_OF_MEMORY, "handle");
   const size_t pt_bytes = 2 * (size_t)c->limbs * 4;
-  if (weighted == 1 && n) {
-    // weighted-point table 2^(ct) P_i for every window t (M = 1)
-    const int W = c->table_windows(n, window_bits);
+  if (weighted >= 1 && n) {
+    // checkpoint table 2^(c M j) P_i (Algorithm 1, interval M = weighted)
+    h->interval = weighted;
+    const int W = c->table_windows(n, window_bits, weighted);
     if ((uint64_t)n * W >= (1ull << 31)) { delete h; return set_error(GZKP_ERROR_INVALID_VALUE, "table >= 2^31 points"); }
     h->bytes = n * W * pt_bytes;
     cudaError_t e = cudaMalloc(&h->pts, h->bytes);
     if (e != cudaSuccess) { delete h; return cuda_status(e, "cudaMalloc(weighted table)"); }
-    gzkp_status st = c->precompute(points_affine, n, window_bits, h->pts, &h->c, &h->W, (cudaStream_t)stream);
+    gzkp_status st = c->precompute(points_affine, n, window_bits, weighted, h->pts, &h->c, &h->W, (cudaStream_t)stream);
     if (st) { cudaFree(h->pts); delete h; return st; }
     h->weighted = true;
   } else if (n) {
@@ -531,7 +534,7 @@ gzkp_status gzkp_prepared_info(const void* handle, int* window_bits, int* window
   if (!h) return set_error(GZKP_ERROR_INVALID_VALUE, "NULL handle");
   if (window_bits) *window_bits = h->c;
   if (windows) *windows = h->W;
-  if (weighted) *weighted = h->weighted ? 1 : 0;
+  if (weighted) *weighted = h->weighted ? h->interval : 0;
   if (bytes) *bytes = h->bytes;
   return GZKP_SUCCESS;
 }
@@ -549,6 +552,7 @@ static gzkp_status msm_prepared_impl(const void* handle, const void* scalars, si
   call.points = h->pts;
   call.prepared = true;
   call.consolidated = h->weighted;
+  call.interval = h->interval;
   call.window_bits = h->c;
   call.table_n = h->n;
   call.scalars = scalars;

@@ -25,7 +25,8 @@ Tunables& tunables();
 struct MsmCall {
   const void* points = nullptr;   // canonical affine, or Montgomery when prepared
   bool prepared = false;
-  bool consolidated = false;      // points = weighted-point table [W][table_n] (NEXT-1)
+  bool consolidated = false;      // points = checkpoint table [ceil(W/interval)][table_n] (NEXT-1)
+  int interval = 1;               // Algorithm 1 checkpoint interval M (consolidated only)
   int window_bits = 0;            // forced c (0 = planner); set for consolidated tables
   size_t table_n = 0;
   cudaEvent_t points_ready = nullptr;   // if set: the accumulation waits for it (overlapped H2D)
@@ -51,8 +52,10 @@ struct CurveImpl {
   gzkp_status (*fixed_base)(const void* scalars, size_t n, void* out, cudaStream_t s);
   gzkp_status (*field_op)(int op, const void* a, const void* b, void* out, size_t n, cudaStream_t s);
   gzkp_status (*ec_op)(int op, const void* P, const void* Q, void* out, size_t n, cudaStream_t s);
-  gzkp_status (*precompute)(const void* in, size_t n, int c, void* table, int* c_out, int* w_out, cudaStream_t s);
-  int (*table_windows)(size_t n, int c);
+  // checkpoint table: copies j < ceil(W / interval) of 2^(c interval j) P_i
+  gzkp_status (*precompute)(const void* in, size_t n, int c, int interval, void* table, int* c_out, int* w_out,
+                            cudaStream_t s);
+  int (*table_windows)(size_t n, int c, int interval);   // copies in the table
   // GZKP_DEBUG_CHECKS: points (canonical, may be null) / scalars (may be null)
   // -> flags (bit 0 coordinate >= p, 1 off curve, 2 scalar >= 2^b); synchronises
   gzkp_status (*validate)(const void* pts, const void* sc, size_t n, uint32_t* flags_host, cudaStream_t s);

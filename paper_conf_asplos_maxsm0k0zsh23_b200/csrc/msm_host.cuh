@@ -26,8 +26,9 @@ namespace gzkp {
 struct Plan {
   int c = 0, W = 0;
   uint32_t B = 0;        // buckets per window = 2^(c-1)
-  bool consolidated = false;   // NEXT-1: windows share one bucket set (weighted points)
-  int Wb = 0;            // bucket windows: W, or 1 when consolidated
+  bool consolidated = false;   // NEXT-1: windows share bucket sets (weighted points, Algorithm 1)
+  int Mi = 0;            // bucket set of window t = t mod Mi: W (standard) or the checkpoint interval M
+  int Wb = 0;            // bucket windows (sets): Mi
   uint32_t val_stride = 0;     // table stride of the weighted points (consolidated)
   uint32_t M = 0;        // Wb * B bucket keys
   int S = 64;            // entries per accumulation chunk
@@ -102,9 +103,10 @@ struct Impl {
     return 15.0 * std::ceil(std::log(q) / std::log((double)HEAVY_SPAN));
   }
 
-  // Window size when all windows share one bucket set (weighted points): no
-  // window combination, reduction over 2^(c-1) buckets once, so larger c pays.
-  static int window_bits_consolidated(size_t n) {
+  // Window size when the windows share M bucket sets (weighted points,
+  // checkpoint interval M): M reductions of 2^(c-1) buckets and (M-1) c
+  // doublings instead of W and (W-1) c, so a larger c pays.
+  static int window_bits_consolidated(size_t n, int interval = 1) {
     if (const char* e = getenv("GZKP_WINDOW_BITS_PREPARED")) {
       int v = atoi(e);
       if (v >= 2 && v <= 22) return v;
@@ -117,8 +119,10 @@ struct Impl {
       const int W = (C::SCALAR_BITS + 1 + c - 1) / c;
       const double B = std::ldexp(1.0, c - 1);
       const double entries = (double)n * W * (1.0 - std::ldexp(1.0, -c));
-      const double reduce = B * 3.4 * add + 60.0 * add * lat / 8.0;
-      const double cost = entries * madd + reduce;
+      const int Mi = std::min(std::max(interval, 1), W);
+      const double reduce = Mi * B * 3.4 * add + 60.0 * add * lat / 8.0;
+      const double tail = (Mi - 1) * (c * 10.0 + add) * lat;
+      const double cost = entries * madd + reduce + tail;
       if (cost < best_cost) { best_cost = cost; best = c; }
     }
     return best;
@@ -183,14 +187,16 @@ struct Impl {
     }
   }
 
-  static Plan plan(size_t n, bool prepared, bool consolidated = false, int c_forced = 0, size_t table_n = 0) {
+  static Plan plan(size_t n, bool prepared, bool consolidated = false, int c_forced = 0, size_t table_n = 0,
+                   int interval = 1) {
     Plan p;
     p.n = n;
     p.consolidated = consolidated;
     p.c = c_forced > 0 ? c_forced : window_bits(n);
     p.W = (C::SCALAR_BITS + 1 + p.c - 1) / p.c;
     p.B = 1u << (p.c - 1);
-    p.Wb = consolidated ? 1 : p.W;
+    p.Mi = consolidated ? std::min(std::max(interval, 1), p.W) : p.W;
+    p.Wb = p.Mi;
     p.val_stride = consolidated ? (uint32_t)table_n : 0u;
     p.M = (uint32_t)p.Wb * p.B;
     int S = tunables().chunk_entries;
@@ -240,7 +246,7 @@ struct Impl {
     uint64_t seg_elems = 1, mid_elems = 1, terms_elems = 1, hlist_elems = 0;
     for (auto& g : p.groups) {
       const uint64_t wins = consolidated ? (uint64_t)p.W : (uint64_t)(g.t_hi - g.t_lo + 1);
-      const uint64_t bwins = consolidated ? 1 : wins;
+      const uint64_t bwins = consolidated ? (uint64_t)p.Mi : wins;
       // reduction segment of this group: <= 16 buckets, fewer until >= 32K threads
       static const uint64_t target = [] {
         const char* e = getenv("GZKP_REDUCE_THREADS");
@@ -338,12 +344,12 @@ struct Impl {
       return GZKP_SUCCESS;
     }
     if ((uint64_t)n >= (1ull << 31)) return set_error(GZKP_ERROR_INVALID_VALUE, "n >= 2^31 not supported");
-    const Plan p = plan(n, call.prepared, call.consolidated, call.window_bits, call.table_n);
+    const Plan p = plan(n, call.prepared, call.consolidated, call.window_bits, call.table_n, call.interval);
     if (p.E_max >= (1ull << 32) - 1) return set_error(GZKP_ERROR_INVALID_VALUE, "n * windows >= 2^32");
     // the bucket-offset scan is two-level: <= SCAN_TILE tiles of SCAN_TILE keys
     if ((uint64_t)p.M > (uint64_t)SCAN_TILE * SCAN_TILE)
       return set_error(GZKP_ERROR_INVALID_VALUE, "too many bucket keys (window bits too large for this curve)");
-    if (p.consolidated && (uint64_t)p.val_stride * p.W >= (1ull << 31))
+    if (p.consolidated && (uint64_t)p.val_stride * ((p.W + p.Mi - 1) / p.Mi) >= (1ull << 31))
       return set_error(GZKP_ERROR_INVALID_VALUE, "weighted-point table >= 2^31 points");
     char* ws = (char*)call.workspace;
     if (!ws) {
@@ -369,8 +375,7 @@ struct Impl {
     GZ_CHECK(cudaMemsetAsync(U(p.o_mcnt), 0, 4 * (p.groups.size() + 1), s));
     GZ_CHECK(cudaMemsetAsync(U(p.o_heavy), 0, 4 * (p.groups.size() + 4), s));
     const uint32_t bpw = (uint32_t)((n + DIGIT_THREADS - 1) / DIGIT_THREADS);
-    const uint32_t key_stride = p.consolidated ? 0u : p.B;
-    k_digits<C><<<bpw, DIGIT_THREADS, 0, s>>>((const uint32_t*)call.scalars, n, p.c, p.W, key_stride, U(p.o_codes),
+    k_digits<C><<<bpw, DIGIT_THREADS, 0, s>>>((const uint32_t*)call.scalars, n, p.c, p.W, p.B, (uint32_t)p.Mi, U(p.o_codes),
                                               U(p.o_counts));
     GZ_CHECK(cudaGetLastError());
     // exclusive scan -> offsets (+ cursor copy); offsets[M] = E
@@ -380,7 +385,7 @@ struct Impl {
     k_scan_add<<<ntiles, SCAN_THREADS, 0, s>>>(U(p.o_offsets), U(p.o_cursor), p.M, U(p.o_tiles));
     // a3: scatter into bucket order (window-major grid)
     const uint32_t bpw_s = (uint32_t)((n + SCATTER_TILE - 1) / SCATTER_TILE);
-    k_scatter<<<(unsigned)((uint64_t)bpw_s * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw_s, key_stride,
+    k_scatter<<<(unsigned)((uint64_t)bpw_s * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw_s, p.B, (uint32_t)p.Mi,
                                                                          p.val_stride, U(p.o_hot), U(p.o_cursor), U(p.o_vals));
     GZ_CHECK(cudaGetLastError());
     *launches += 5;
@@ -613,7 +618,7 @@ struct Impl {
       launches += 2 + gr.heavy_levels;
       ev_merged = profile_event(prof, ss);
       // a6 (side stream): bucket reduction of the group's windows
-      const int gw = p.consolidated ? 1 : gr.t_hi - gr.t_lo + 1;
+      const int gw = p.consolidated ? p.Wb : gr.t_hi - gr.t_lo + 1;
       const int t_lo = p.consolidated ? 0 : gr.t_lo;
       const uint32_t G = p.B / gr.seg;
       const uint32_t total = (uint32_t)gw * G;
@@ -643,7 +648,7 @@ struct Impl {
       ev_reduced = profile_event(prof, ss);
       // a7 (+ a8 on the last group): Horner over the group's windows
       const int last = gi == ngroups - 1;
-      k_tail<C><<<1, 32, 0, ss>>>(U(p.o_win), p.consolidated ? 0 : gr.t_hi, t_lo, p.c, gi == 0, last, U(p.o_state),
+      k_tail<C><<<1, 32, 0, ss>>>(U(p.o_win), p.consolidated ? p.Wb - 1 : gr.t_hi, t_lo, p.c, gi == 0, last, U(p.o_state),
                                   last ? (uint32_t*)call.out_partial : nullptr,
                                   last ? (uint32_t*)call.out_affine : nullptr);
       GZ_CHECK(cudaGetLastError());
@@ -662,28 +667,35 @@ struct Impl {
     return GZKP_SUCCESS;
   }
 
-  // NEXT-1 prepare: table[t*n + i] = 2^(ct) P_i (Montgomery affine), t < W.
-  // Returns the window bits used (the MSM calls on this table must use them).
-  static gzkp_status precompute(const void* in, size_t n, int c, void* table, int* c_out, int* w_out, cudaStream_t s) {
-    if (c <= 0) c = window_bits_consolidated(n);
-    const int W = (C::SCALAR_BITS + 1 + c - 1) / c;
+  // NEXT-1 prepare (Algorithm 1): the checkpoint table
+  // table[j*n + i] = 2^(c M j) P_i (Montgomery affine), j < ceil(W / M), for
+  // checkpoint interval M (M = 1: every window's weighted copy).  Returns the
+  // window bits and the number of copies (the MSMs on this table use them).
+  static gzkp_status precompute(const void* in, size_t n, int c, int interval, void* table, int* c_out, int* w_out,
+                                cudaStream_t s) {
+    if (c <= 0) c = window_bits_consolidated(n, interval);
+    const int copies = table_windows(n, c, interval);
+    const int M = std::min(std::max(interval, 1), (C::SCALAR_BITS + 1 + c - 1) / c);
     *c_out = c;
-    *w_out = W;
+    *w_out = copies;
     if (!n) return GZKP_SUCCESS;
     uint32_t* T = (uint32_t*)table;
     if (gzkp_status st = to_mont(in, T, n, s)) return st;
     const int threads = 128;
     const int grid = (int)std::min<size_t>((n + threads - 1) / threads, (size_t)device_sm_count() * 32);
-    for (int t = 1; t < W; ++t) {
-      k_precompute_step<C><<<grid, threads, 0, s>>>(T + (size_t)(t - 1) * n * 2 * N, T + (size_t)t * n * 2 * N, n, c);
+    for (int j = 1; j < copies; ++j) {
+      k_precompute_step<C><<<grid, threads, 0, s>>>(T + (size_t)(j - 1) * n * 2 * N, T + (size_t)j * n * 2 * N, n,
+                                                    c * M);
       GZ_CHECK(cudaGetLastError());
     }
     return GZKP_SUCCESS;
   }
 
-  static int table_windows(size_t n, int c) {
-    if (c <= 0) c = window_bits_consolidated(n);
-    return (C::SCALAR_BITS + 1 + c - 1) / c;
+  static int table_windows(size_t n, int c, int interval) {
+    if (c <= 0) c = window_bits_consolidated(n, interval);
+    const int W = (C::SCALAR_BITS + 1 + c - 1) / c;
+    const int M = std::min(std::max(interval, 1), W);
+    return (W + M - 1) / M;
   }
 
   static gzkp_status combine(const void* partials, int count, void* out, cudaStream_t s) {

@@ -129,9 +129,11 @@ GZ_DEV int hot_slot(uint32_t* s_key, uint32_t key) {
 constexpr int DIGIT_THREADS = 256;
 constexpr uint32_t DIG_SMALL = 16;
 constexpr int DIG_SMALL_WIN = 64;             // small table: W <= 64 windows
+// Bucket set of window t: t mod Mi (Mi = W: one set per window, standard;
+// Mi = M: the checkpoint interval of GZKP's Algorithm 1, weighted points).
 template <class C>
 __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __restrict__ sc, size_t n, int c, int W,
-                                                          uint32_t key_stride, uint32_t* __restrict__ codes,
+                                                          uint32_t B, uint32_t Mi, uint32_t* __restrict__ codes,
                                                           uint32_t* __restrict__ counts) {
   constexpr int NS = C::NS;
   __shared__ uint32_t s_sc[NS * DIGIT_THREADS];
@@ -154,11 +156,12 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
   const size_t i = base + tid;
   auto word = [&](int w) -> uint32_t { return w < NS ? s_sc[w * DIGIT_THREADS + tid] : 0u; };
   const int lane = tid & 31;
-  for (int t = 0; t < W; ++t) {
+  uint32_t tr = 0;                                     // t mod Mi
+  for (int t = 0; t < W; ++t, tr = tr + 1 == Mi ? 0u : tr + 1) {
     const uint32_t code = live ? digit_code(booth_digit(word, t, c)) : 0u;
     if (live) codes[(size_t)t * n + i] = code;
     const uint32_t mag = code & ~VAL_NEG;
-    const uint32_t key = (uint32_t)t * key_stride + mag - 1u;
+    const uint32_t key = tr * B + mag - 1u;
     const bool small = code && use_small && mag <= DIG_SMALL;
     if (__any_sync(0xffffffffu, small) && small) {       // skewed inputs: many lanes share a small digit
       const unsigned peers = __match_any_sync(__activemask(), mag);
@@ -187,13 +190,14 @@ __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __rest
   if (tid < HOT_SLOTS && s_key[tid] != HOT_EMPTY) atomicAdd(&counts[s_key[tid]], s_cnt[tid]);
   if (use_small)
     for (int q = tid; q < W * (int)DIG_SMALL; q += DIGIT_THREADS)
-      if (s_small[q]) atomicAdd(&counts[(uint32_t)(q / DIG_SMALL) * key_stride + q % DIG_SMALL], s_small[q]);
+      if (s_small[q]) atomicAdd(&counts[(uint32_t)(q / DIG_SMALL) % Mi * B + q % DIG_SMALL], s_small[q]);
 }
 
-// Cross-window consolidation (§4.1; NEXT-1): with prepared
-// weighted points P_{i,t} = 2^(ct) P_i stored as table[t*n + i], every window
-// uses the SAME bucket set: key_stride = 0 and the entry value indexes the
-// table (val_stride = n).  Without it key_stride = B, val_stride = 0.
+// Cross-window consolidation (§4.1, Algorithm 1; NEXT-1):
+// with checkpoints P_{i,j} = 2^(c M j) P_i stored as table[j*n + i] (interval
+// M), window t = M j + r uses checkpoint j and bucket set r: key = r B + |d| - 1,
+// val = j n + i (val_stride = n).  M = 1 is the full weighted table (one
+// bucket set); the standard pipeline is Mi = W, val_stride = 0.
 // ------------------------------------------------------ a3 scatter (sort)
 // Window-major 1-D grid (block b covers window b / bpw) so the blocks in
 // flight write into one or two windows' 4n-byte ranges, which stay resident in
@@ -211,7 +215,7 @@ constexpr int SCATTER_TILE = SCATTER_THREADS * SCATTER_PER_THREAD;
 // one returning atomic (same-address contention <= HOT_COUNT per key).
 constexpr uint32_t HOT_COUNT = 1024;
 static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32_t* __restrict__ codes, size_t n,
-                                                             uint32_t bpw, uint32_t key_stride, uint32_t val_stride,
+                                                             uint32_t bpw, uint32_t B, uint32_t Mi, uint32_t val_stride,
                                                              const uint32_t* __restrict__ hotbits,
                                                              uint32_t* __restrict__ cursor, uint32_t* __restrict__ vals) {
   __shared__ uint32_t s_key[HOT_SLOTS], s_cnt[HOT_SLOTS], s_base[HOT_SLOTS];
@@ -219,6 +223,7 @@ static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32
   if (tid < HOT_SLOTS) { s_key[tid] = HOT_EMPTY; s_cnt[tid] = 0; }
   __syncthreads();
   const uint32_t t = blockIdx.x / bpw;
+  const uint32_t kbase = t % Mi * B, vbase = t / Mi * val_stride;
   const size_t i0 = (size_t)(blockIdx.x % bpw) * SCATTER_TILE + (size_t)tid * SCATTER_PER_THREAD;
   const uint32_t* crow = codes + (size_t)t * n;
   uint32_t code[SCATTER_PER_THREAD];
@@ -238,7 +243,7 @@ static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32
 #pragma unroll
   for (int q = 0; q < SCATTER_PER_THREAD; ++q) {
     peers[q] = 0; leader[q] = 0; h[q] = -1; pos[q] = 0;
-    const uint32_t key = t * key_stride + (code[q] & ~VAL_NEG) - 1u;
+    const uint32_t key = kbase + (code[q] & ~VAL_NEG) - 1u;
     hot[q] = code[q] && ((__ldg(hotbits + (key >> 5)) >> (key & 31)) & 1u);
     if (code[q] && !hot[q]) pos[q] = atomicAdd(&cursor[key], 1u);
     any_hot |= hot[q];
@@ -246,7 +251,7 @@ static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32
   if (__syncthreads_or(any_hot)) {
 #pragma unroll
     for (int q = 0; q < SCATTER_PER_THREAD; ++q) {
-      const uint32_t key = t * key_stride + (code[q] & ~VAL_NEG) - 1u;
+      const uint32_t key = kbase + (code[q] & ~VAL_NEG) - 1u;
       if (!__any_sync(0xffffffffu, hot[q])) continue;
       if (hot[q]) {
         peers[q] = __match_any_sync(__activemask(), key);
@@ -271,7 +276,7 @@ static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32
         if (lane == leader[q] && h[q] >= 0) p += s_base[h[q]];
         p = __shfl_sync(peers[q], p, leader[q]) + __popc(peers[q] & ((1u << lane) - 1u));
       }
-      vals[p] = (t * val_stride + (uint32_t)(i0 + q)) | (code[q] & VAL_NEG);
+      vals[p] = (vbase + (uint32_t)(i0 + q)) | (code[q] & VAL_NEG);
     }
   }
 }

@@ -58,10 +58,12 @@ def test_closed_form_full_size(curve, log_n, cfg, dist):
     got, _ = _msm_checked(gz, curve, pts, dev(k), n)
     want = oracle.closed_form(curve, k, d)
     assert np.array_equal(got, want)
-    # the same MSM through prepared weighted points (NEXT-1), planner's c
-    h = gz.PreparedPoints(curve, pts, weighted=True)
-    assert np.array_equal(host(h.msm(dev(k))), want)
-    h.release()
+    # the same MSM through prepared weighted points (NEXT-1), planner's c,
+    # full table (M = 1) and Algorithm 1 checkpoints (M = 2, 3)
+    for M in (1, 2, 3):
+        h = gz.PreparedPoints(curve, pts, weighted=M)
+        assert np.array_equal(host(h.msm(dev(k))), want), M
+        h.release()
 
 
 @pytest.mark.parametrize("curve,log_n,cfg,dist,tile_log", [

@@ -263,3 +263,33 @@ def test_heavy_buckets_tree(curve):
             gz.set_config(0, chunk)
             assert np.array_equal(run(gz, curve, pts, k), want), chunk
     gz.set_config(0, 0)
+
+
+@pytest.mark.parametrize("curve,c,intervals", [("bn254", 16, (2, 3, 5, 16, 40)), ("bls12_381", 13, (2, 4, 20)),
+                                               ("bls12_381", 20, (2, 3)), ("mnt4_753", 11, (2, 7, 69)),
+                                               ("toy_a2", 3, (2, 5)), ("toy_a0", 2, (3, 8))])
+def test_checkpoint_interval_algorithm1(curve, c, intervals):
+    """GZKP's Algorithm 1 with checkpoint interval M > 1:
+    only the checkpoints 2^(c M j) P_i are stored and window t = M j + r
+    accumulates checkpoint j into bucket set r (reading R10).  Bit-exact vs the
+    oracle for several M, including M >= W (no table: the standard pipeline),
+    sparse scalars, an identity input and a prefix of the prepared vector."""
+    gz = require_cuda()
+    n = 64 if curve == "mnt4_753" else 1024
+    pts, _ = oracle_points(curve, n)
+    pts = pts.copy()
+    pts[7] = 0
+    c_ = curves.get(curve)
+    W = -(-(c_.scalar_bits + 1) // c)
+    for dist in ("uniform", "zcash_like") if curve != "mnt4_753" else ("uniform",):
+        k = synth.scalars(curve, n, 52, dist)
+        want = oracle_msm_cached(curve, pts, k)
+        want_prefix = oracle_msm_cached(curve, pts[:n // 2], k[:n // 2])
+        for M in intervals:
+            h = gz.PreparedPoints(curve, dev(pts), weighted=M, window_bits=c)
+            info = h.info()
+            Mi = min(M, W)
+            assert info["interval"] == M and info["windows"] == -(-W // Mi), info
+            assert np.array_equal(host(h.msm(dev(k))), want), (dist, M)
+            assert np.array_equal(host(h.msm(dev(k[:n // 2]))), want_prefix), (dist, M)
+            h.release()
