@@ -213,7 +213,9 @@ gzkp_status gzkp_debug_buckets(int curve, const void *scalars, size_t n, int win
  * NEXT-2, measured slower than the IMAD product and off by default); every
  * other curve, MNT4-753 included, computes op 6 with the IMAD product,
  * 7: a^-1 mod p by the constant-time binary GCD (the batch-affine inverse;
- * G2 curves fall back to op 3).  For G2 curves the elements are F_p^2 values
+ * G2 curves fall back to op 3), 8: a*b mod p by the lane-split product of the
+ * cooperative chains (8 lanes per product, BN254 / BLS12-381 / MNT4-753; other
+ * curves: the one-thread product).  For G2 curves the elements are F_p^2 values
  * c0 || c1. */
 gzkp_status gzkp_field_op(int curve, int op, const void *a, const void *b, void *out, size_t n,
                           gzkp_stream stream);

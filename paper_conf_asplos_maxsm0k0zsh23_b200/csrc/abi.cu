@@ -607,7 +607,7 @@ gzkp_status gzkp_field_op(int curve, int op, const void* a, const void* b, void*
   init_pool_once();
   const CurveImpl* c = impl_for(curve);
   if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
-  if (op < 0 || op > 7 || (n && (!a || !b || !out))) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
+  if (op < 0 || op > 8 || (n && (!a || !b || !out))) return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
   return c->field_op(op, a, b, out, n, (cudaStream_t)stream);
 }
 

@@ -16,6 +16,11 @@
 #include "field.cuh"
 #include "field2.cuh"
 #include "field_dfp.cuh"
+#include "coop_mul.cuh"
+
+#ifndef GZKP_COOP_SPLIT
+#define GZKP_COOP_SPLIT 0   // 1: lane-split products (coop_mul.cuh) in the cooperative chains
+#endif
 
 #ifndef GZKP_COOP_KARATSUBA
 #define GZKP_COOP_KARATSUBA 0   // 1: Karatsuba products in the cooperative chains (measured slower: BLS12-381 tail 1.01 -> 1.20 ms)
@@ -252,9 +257,20 @@ struct CoopEC {
   using E = EC<C>;
   using Xyzz = typename E::Xyzz;
 
+  // lane-split products (coop_mul.cuh): product q of a level is computed by
+  // lanes 8q .. 8q+7 and published in shared memory; otherwise lane q
+  // computes it alone and it is broadcast by shuffles
+  // GZKP_COOP_SPLIT=1 (compile time): measured slower than the one-lane
+  // product (BLS12-381 tail 1.00 -> 1.55 ms, MNT4-753 2^17 10.97 -> 11.19 ms;
+  // profiles/r02_coop_split_experiment.md), so off by default
+  static constexpr bool SPLIT = GZKP_COOP_SPLIT && CoopMul<C>::ON && std::is_same<Fp, F<C>>::value;
   GZ_DEV static void bcast(uint32_t d[N], const uint32_t s[N], int src) {
+    if constexpr (SPLIT) {
+      CoopMul<C>::result(d, src);
+    } else {
 #pragma unroll
-    for (int i = 0; i < N; ++i) d[i] = __shfl_sync(0xffffffffu, s[i], src);
+      for (int i = 0; i < N; ++i) d[i] = __shfl_sync(0xffffffffu, s[i], src);
+    }
   }
   // branch-free 4-way blend by lane (pure LOP3s: no local-memory indexing)
   GZ_DEV static void pick(uint32_t d[N], int q, const uint32_t* a0, const uint32_t* a1, const uint32_t* a2,
@@ -268,10 +284,14 @@ struct CoopEC {
   GZ_DEV static void level(uint32_t r[N], const uint32_t* x0, const uint32_t* y0, const uint32_t* x1,
                            const uint32_t* y1, const uint32_t* x2, const uint32_t* y2, const uint32_t* x3,
                            const uint32_t* y3) {
-    const int q = threadIdx.x & 3;
+    const int q = SPLIT ? (threadIdx.x & 31) >> 3 : threadIdx.x & 3;
     uint32_t x[N], y[N];
     pick(x, q, x0, x1, x2, x3);
     pick(y, q, y0, y1, y2, y3);
+    if constexpr (SPLIT) {
+      CoopMul<C>::mul(r, x, y, CoopMul<C>::smem());
+      return;
+    }
     // always inlined here (also for N = 24): per-lane operands feeding an
     // out-of-line call between warp shuffles produced wrong MNT4-753 results.
     // GZKP_COOP_KARATSUBA=1 tries the one-level Karatsuba product here (three

@@ -715,6 +715,12 @@ struct Impl {
 
   static gzkp_status field_op(int op, const void* a, const void* b, void* out, size_t n, cudaStream_t s) {
     if (!n) return GZKP_SUCCESS;
+    if (op == 8) {
+      const int grid = (int)std::min<size_t>((n + 3) / 4, (size_t)device_sm_count() * 32);
+      k_coop_mul_test<C><<<grid, 32, 0, s>>>((const uint32_t*)a, (const uint32_t*)b, (uint32_t*)out, n);
+      GZ_CHECK(cudaGetLastError());
+      return GZKP_SUCCESS;
+    }
     const int threads = 128;
     const int grid = (int)std::min<size_t>((n + threads - 1) / threads, 4096);
     k_field_op<C><<<grid, threads, 0, s>>>(op, (const uint32_t*)a, (const uint32_t*)b, (uint32_t*)out, n);

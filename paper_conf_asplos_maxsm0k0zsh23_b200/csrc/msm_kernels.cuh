@@ -1025,6 +1025,28 @@ __global__ void k_field_op(int op, const uint32_t* __restrict__ a, const uint32_
   }
 }
 
+// field op 8: the lane-split Montgomery product (coop_mul.cuh) on canonical
+// inputs; one warp per CTA, lanes 8g .. 8g+7 multiply element base + g
+template <class C>
+__global__ void __launch_bounds__(32) k_coop_mul_test(const uint32_t* __restrict__ a, const uint32_t* __restrict__ b,
+                                                      uint32_t* __restrict__ out, size_t n) {
+  using Fp = Field<C>;
+  constexpr int N = C::N;
+  const int lane = threadIdx.x & 31, g = lane >> 3;
+  for (size_t base = (size_t)blockIdx.x * 4; base < n; base += (size_t)gridDim.x * 4) {
+    const size_t e = base + g < n ? base + g : n - 1;        // uniform control flow: clamp
+    uint32_t x[N], y[N], r[N];
+    EC<C>::ld(x, a + e * N);
+    EC<C>::ld(y, b + e * N);
+    Fp::to_mont(x, x);
+    Fp::to_mont(y, y);
+    if constexpr (CoopMul<C>::ON && std::is_same<Fp, F<C>>::value) CoopMul<C>::mul(r, x, y, CoopMul<C>::smem());
+    else Fp::mul(r, x, y);
+    Fp::from_mont(r, r);
+    if ((lane & 7) == 0 && base + g < n) EC<C>::st(out + e * N, r);
+  }
+}
+
 template <class C>
 __global__ void k_ec_op(int op, const uint32_t* __restrict__ P, const uint32_t* __restrict__ Q,
                         uint32_t* __restrict__ out, size_t n) {

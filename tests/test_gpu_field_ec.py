@@ -47,10 +47,12 @@ def test_field_ops(c):
     rt = host(gz.field_op(c.name, 4, A, B))
     sq = host(gz.field_op(c.name, 5, A, B))
     dfp = host(gz.field_op(c.name, 6, A, B))       # FP64 (DFP) product where available
+    coop = host(gz.field_op(c.name, 8, A, B))      # lane-split product (8 lanes per product)
     for i in range(len(a)):
         assert limbs_int(sq[i]) == a[i] * a[i] % c.p, (i, a[i])
         assert limbs_int(dfp[i]) == a[i] * b[i] % c.p, ("dfp", i, a[i], b[i])
         assert limbs_int(mul[i]) == a[i] * b[i] % c.p, (i, a[i], b[i])
+        assert limbs_int(coop[i]) == a[i] * b[i] % c.p, ("coop", i, a[i], b[i])
         assert limbs_int(add[i]) == (a[i] + b[i]) % c.p, i
         assert limbs_int(sub[i]) == (a[i] - b[i]) % c.p, i
         assert limbs_int(rt[i]) == a[i], i

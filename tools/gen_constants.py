@@ -170,6 +170,7 @@ def main():
                    f"  GZ_HD static constexpr uint32_t ONE(int i) {{ constexpr uint32_t v[N] = {arr(R % p, n)}; return v[i]; }}  // R mod p\n"
                    f"  GZ_HD static constexpr uint32_t R2(int i) {{ constexpr uint32_t v[N] = {arr(R * R % p, n)}; return v[i]; }}  // R^2 mod p\n"
                    f"  GZ_HD static constexpr uint32_t A_MONT(int i) {{ constexpr uint32_t v[N] = {arr(a * R % p, n)}; return v[i]; }}\n"
+                   f"  GZ_HD static constexpr uint32_t NP(int i) {{ constexpr uint32_t v[N] = {arr((-pow(p, -1, R)) % R, n)}; return v[i]; }}  // -p^-1 mod R\n"
                    f"  GZ_HD static constexpr uint32_t GX(int i) {{ constexpr uint32_t v[N] = {arr(gx, n)}; return v[i]; }}  // generator, canonical\n"
                    f"  GZ_HD static constexpr uint32_t GY(int i) {{ constexpr uint32_t v[N] = {arr(gy, n)}; return v[i]; }}\n"
                    + dfp_block(p, n) +
