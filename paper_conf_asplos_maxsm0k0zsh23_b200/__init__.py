@@ -15,7 +15,8 @@ from typing import Optional
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libgzkp.so")
+# GZKP_LIB: an experiment build of the same library (build.py -D... --out ...)
+LIB_PATH = os.environ.get("GZKP_LIB") or os.path.join(_HERE, "libgzkp.so")
 
 CURVES = {"bn254": 0, "bls12_381": 1, "mnt4_753": 2, "toy_a0": 100, "toy_a2": 101,
           "bn254_g2": 3, "bls12_381_g2": 4}

@@ -50,9 +50,9 @@ def _deps(obj: str, src: str):
         return _headers() + [src]
 
 
-def _compile(src: str, verbose: bool) -> str:
-    obj = os.path.join(BUILD, os.path.basename(src)[:-3] + ".o")
-    cmd = [NVCC, *ARCH, *FLAGS, "-MD", "-MF", obj[:-2] + ".d", "-c", src, "-o", obj]
+def _compile(src: str, verbose: bool, build_dir: str = BUILD, defines=()) -> str:
+    obj = os.path.join(build_dir, os.path.basename(src)[:-3] + ".o")
+    cmd = [NVCC, *ARCH, *FLAGS, *[f"-D{d}" for d in defines], "-MD", "-MF", obj[:-2] + ".d", "-c", src, "-o", obj]
     if verbose:
         cmd += ["-Xptxas", "-v"]
     r = subprocess.run(cmd, capture_output=True, text=True)
@@ -63,33 +63,37 @@ def _compile(src: str, verbose: bool) -> str:
     return obj
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, defines=(), lib: str = LIB) -> str:
     """Recompile each translation unit whose object is older than the source or
     any header in its depfile (headers edited while a build runs are caught:
     the check is per object, never "library newer than the sources"), then
     relink if any object is newer than the library."""
     srcs = _sources()
-    os.makedirs(BUILD, exist_ok=True)
+    build_dir = BUILD if not defines else BUILD + "_" + "_".join(d.replace("=", "") for d in defines)
+    os.makedirs(build_dir, exist_ok=True)
     todo = []
     objs = []
     for s in srcs:
-        obj = os.path.join(BUILD, os.path.basename(s)[:-3] + ".o")
+        obj = os.path.join(build_dir, os.path.basename(s)[:-3] + ".o")
         objs.append(obj)
         if force or verbose or not os.path.exists(obj) or os.path.getmtime(obj) < _newest(_deps(obj, s)):
             todo.append(s)
     if todo:
         with cf.ThreadPoolExecutor(max_workers=max(1, min(len(todo), os.cpu_count() or 4))) as ex:
-            list(ex.map(lambda s: _compile(s, verbose), todo))
-    if not todo and os.path.exists(LIB) and os.path.getmtime(LIB) >= _newest(objs):
-        return LIB
-    tmp = LIB + ".tmp.%d" % os.getpid()
+            list(ex.map(lambda s: _compile(s, verbose, build_dir, defines), todo))
+    if not todo and os.path.exists(lib) and os.path.getmtime(lib) >= _newest(objs):
+        return lib
+    tmp = lib + ".tmp.%d" % os.getpid()
     cmd = [NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-lcudart", "-ldl"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
-    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv))
+    # experiment builds: python -m ...build -DGZKP_COOP_SOS=1 --out path/libgzkp_x.so
+    defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
+    out = sys.argv[sys.argv.index("--out") + 1] if "--out" in sys.argv else LIB
+    print(build(force="--force" in sys.argv, verbose="--verbose" in sys.argv, defines=defs, lib=out))

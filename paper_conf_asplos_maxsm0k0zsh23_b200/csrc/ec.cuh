@@ -18,6 +18,10 @@
 #include "field_dfp.cuh"
 #include "coop_mul.cuh"
 
+#ifndef GZKP_COOP_SOS
+#define GZKP_COOP_SOS 0     // 1: separated-operand-scanning products in the cooperative chains
+#endif
+
 #ifndef GZKP_COOP_SPLIT
 #define GZKP_COOP_SPLIT 0   // 1: lane-split products (coop_mul.cuh) in the cooperative chains
 #endif
@@ -298,6 +302,9 @@ struct CoopEC {
     // independent half products for the single warp's ILP): measured slower.
 #if GZKP_COOP_KARATSUBA
     if constexpr (N >= 8 && N <= 12 && N % 4 == 0) Fp::mul_kara(r, x, y);
+    else Fp::mul_inline(r, x, y);
+#elif GZKP_COOP_SOS
+    if constexpr (N >= 8 && std::is_same<Fp, F<C>>::value) Fp::mul_sos(r, x, y);
     else Fp::mul_inline(r, x, y);
 #else
     Fp::mul_inline(r, x, y);

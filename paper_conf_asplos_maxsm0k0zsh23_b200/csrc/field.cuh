@@ -19,6 +19,10 @@
 #pragma once
 #include <cstdint>
 
+#ifndef GZKP_MUL_SOS
+#define GZKP_MUL_SOS 0         // 1: separated-operand-scanning products everywhere (experiment)
+#endif
+
 #ifndef GZKP_MUL_KARATSUBA
 #define GZKP_MUL_KARATSUBA 0   // 1: one-level Karatsuba products (N % 4 == 0; measured slower, see mul_kara)
 #endif
@@ -136,7 +140,21 @@ struct F {
 #pragma unroll
     for (int i = 0; i < N; ++i) r[i] = z[i];
   }
+  // separated operand scanning: the full product (prod<N>, parity-split
+  // chains) then sos_reduce; the same 2N^2 + N(2N + 1) IMAD as CIOS, a
+  // different dependency structure (GZKP_MUL_SOS experiment)
+  GZ_DEV static void mul_sos(uint32_t r[N], const uint32_t a[N], const uint32_t b[N]) {
+    uint32_t T[2 * N];
+    prod<N>(T, a, b);
+    sos_reduce(r, T);
+  }
   GZ_DEV static void mul_inline(uint32_t r[N], const uint32_t a[N], const uint32_t b[N]) {
+#if GZKP_MUL_SOS
+    if constexpr (N >= 8) {
+      mul_sos(r, a, b);
+      return;
+    }
+#endif
 #if GZKP_MUL_KARATSUBA
     if constexpr (N >= 8 && N % 4 == 0) {
       mul_kara(r, a, b);
