@@ -236,6 +236,7 @@ gzkp_status stream_ctx(cudaStream_t s, StreamCtx** out) {
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);      // hi = greatest priority
     cudaError_t e = cudaStreamCreateWithPriority(&n->side, cudaStreamNonBlocking, hi);
+    if (e == cudaSuccess) e = cudaStreamCreateWithPriority(&n->side2, cudaStreamNonBlocking, hi);
     if (e != cudaSuccess) { delete n; return cuda_status(e, "cudaStreamCreateWithPriority"); }
     n->nev = 64;
     for (int i = 0; i < n->nev; ++i) cudaEventCreateWithFlags(&n->ev[i], cudaEventDisableTiming);
@@ -261,8 +262,10 @@ static gzkp_status release_stream(cudaStream_t s) {
   if (it != g_ctx.end()) {
     StreamCtx* c = it->second;
     cudaStreamSynchronize(c->side);
+    cudaStreamSynchronize(c->side2);
     for (int i = 0; i < c->nev; ++i) cudaEventDestroy(c->ev[i]);
     cudaStreamDestroy(c->side);
+    cudaStreamDestroy(c->side2);
     delete c;
     g_ctx.erase(it);
   }

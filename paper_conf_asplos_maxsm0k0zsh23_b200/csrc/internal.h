@@ -102,7 +102,8 @@ void profile_end(ProfileRecord* r, const uint32_t* entries_dev, int launches, in
 // per (device, caller stream): a high-priority side stream and reusable
 // sync events for the window-group pipeline
 struct StreamCtx {
-  cudaStream_t side = nullptr;
+  cudaStream_t side = nullptr;    // merge + bucket reduction of the window groups
+  cudaStream_t side2 = nullptr;   // window combination (Horner), group after group
   cudaEvent_t ev[64];
   int nev = 0;
 };

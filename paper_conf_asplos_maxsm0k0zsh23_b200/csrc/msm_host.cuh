@@ -227,9 +227,15 @@ struct Impl {
     } else if (consolidated) {
       p.groups.push_back({0, p.W - 1, 0, p.B, 0, 0, 0, 0, 0});
     } else if (pipeline == 2 && p.W >= 2) {
-      // two equal groups: the top half's merge / reduction / Horner run on the
-      // side stream while the bottom half accumulates
-      const int mid = p.W / 2;
+      // two groups: the top windows' merge / reduction / Horner run on the
+      // side stream while the bottom `low` windows accumulate (equal halves
+      // unless GZKP_PIPELINE_LOW sets the bottom group's size)
+      static const int low_env = [] {
+        const char* e = getenv("GZKP_PIPELINE_LOW");
+        return e ? atoi(e) : 0;
+      }();
+      const int low = low_env > 0 ? std::min(low_env, p.W - 1) : p.W / 2;
+      const int mid = low;
       p.groups.push_back({mid, p.W - 1, (uint32_t)mid * p.B, (uint32_t)p.W * p.B, 0, 0, 0, 0, 0});
       p.groups.push_back({0, mid - 1, 0, (uint32_t)mid * p.B, 0, 0, 0, 0, 0});
     } else {
@@ -493,11 +499,12 @@ struct Impl {
     // while group g+1 accumulates.  One group (weighted points): no side stream.
     const int ngroups = (int)p.groups.size();
     StreamCtx* ctx = nullptr;
-    cudaStream_t ss = s;
+    cudaStream_t ss = s, st2 = s;
     if (ngroups > 1) {
       if (gzkp_status st = stream_ctx(s, &ctx)) return st;
-      if (2 * ngroups + 1 > ctx->nev) return set_error(GZKP_ERROR_INVALID_VALUE, "too many window groups");
+      if (ngroups > 16) return set_error(GZKP_ERROR_INVALID_VALUE, "too many window groups");
       ss = ctx->side;
+      st2 = ctx->side2;
     }
     const int threads = 128;
     // accumulation CTA size: small CTAs let the register file hold more warps
@@ -646,22 +653,30 @@ struct Impl {
       GZ_CHECK(cudaGetLastError());
       launches += 4;
       ev_reduced = profile_event(prof, ss);
-      // a7 (+ a8 on the last group): Horner over the group's windows
+      // a7 (+ a8 on the last group): Horner over the group's windows, on its
+      // own stream so the next group's merge / reduction never queue behind
+      // this latency-bound chain (the chain itself runs group after group)
+      if (ctx) {
+        GZ_CHECK(cudaEventRecord(ctx->ev[16 + gi], ss));
+        GZ_CHECK(cudaStreamWaitEvent(st2, ctx->ev[16 + gi], 0));
+      }
       const int last = gi == ngroups - 1;
-      k_tail<C><<<1, 32, 0, ss>>>(U(p.o_win), p.consolidated ? p.Wb - 1 : gr.t_hi, t_lo, p.c, gi == 0, last, U(p.o_state),
+      k_tail<C><<<1, 32, 0, st2>>>(U(p.o_win), p.consolidated ? p.Wb - 1 : gr.t_hi, t_lo, p.c, gi == 0, last, U(p.o_state),
                                   last ? (uint32_t*)call.out_partial : nullptr,
                                   last ? (uint32_t*)call.out_affine : nullptr);
       GZ_CHECK(cudaGetLastError());
       ++launches;
-      ev_tailed = profile_event(prof, ss);
+      ev_tailed = profile_event(prof, st2);
     }
     // phases 2-4 = the exposed post-processing of the last group
     profile_interval(prof, 2, ev_last_acc, ev_merged);
     profile_interval(prof, 3, ev_merged, ev_reduced);
     profile_interval(prof, 4, ev_reduced, ev_tailed);
-    if (ctx) {   // join: later work on the caller's stream follows the side stream
+    if (ctx) {   // join: later work on the caller's stream follows both side streams
       GZ_CHECK(cudaEventRecord(ctx->ev[ctx->nev - 1], ss));
       GZ_CHECK(cudaStreamWaitEvent(s, ctx->ev[ctx->nev - 1], 0));
+      GZ_CHECK(cudaEventRecord(ctx->ev[ctx->nev - 4], st2));
+      GZ_CHECK(cudaStreamWaitEvent(s, ctx->ev[ctx->nev - 4], 0));
     }
     profile_end(prof, U(p.o_offsets) + p.M, launches, p.c, s);
     return GZKP_SUCCESS;
