@@ -1,10 +1,13 @@
 #!/bin/bash
-# Round bench lines: the default (full contract) and every BASELINE workload.
+# Round bench lines: the default (full contract) and every BASELINE workload,
+# each with the parity leg (closed-form check of the timed MSM's bytes).
 cd "${GRAFT_REPO_ROOT:-/root/repo}"
-mkdir -p gpurun_out/bench
-timeout 300 python bench.py > gpurun_out/bench/default.json 2> gpurun_out/bench/default.err
-for w in bn254_2p20 mnt4_753_2p20 bls12_381_2p26_sparse bls12_381_2p19 bn254_g2_2p20 bls12_381_g2_2p20 bls12_381_2p26; do
-  timeout 300 python bench.py --workload $w --no-cpu-baseline > gpurun_out/bench/$w.json 2> gpurun_out/bench/$w.err
+OUT=${OUT:-gpurun_out/bench}
+mkdir -p $OUT
+timeout 400 python bench.py > $OUT/default.json 2> $OUT/default.err
+for w in bn254_2p10 bn254_2p20 mnt4_753_2p20 mnt4_753_2p17 bls12_381_2p19 bls12_381_2p26_sparse bls12_381_2p26 \
+         bn254_g2_2p20 bls12_381_g2_2p20 bls12_381_ntt_2p24 bn254_ntt_2p22 mnt4_753_ntt_2p20; do
+  timeout 600 python bench.py --workload $w > $OUT/$w.json 2> $OUT/$w.err
 done
-timeout 200 python bench.py --impl reference --steps 2 --warmup 1 > gpurun_out/bench/reference.json 2> gpurun_out/bench/reference.err
-timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/bench/launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-prepared > /dev/null 2>&1
+timeout 300 python bench.py --impl reference --steps 2 --warmup 1 > $OUT/reference.json 2> $OUT/reference.err
+timeout 300 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $OUT/launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline --no-e2e --no-prepared > /dev/null 2>&1
