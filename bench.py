@@ -144,18 +144,23 @@ class ClockSampler:
                 "samples": len(sm)}
 
 
+def relaunch_cmd(nproc: int, argv, port: int):
+    """The torch.distributed.run command line that re-runs this bench with
+    `nproc` ranks on this node (one per GPU, rendezvous on 127.0.0.1)."""
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
+            "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + list(argv)
+
+
 def relaunch_distributed(nproc: int) -> int:
     """`python bench.py --gpus N` without a launcher: re-run this command under
-    torch.distributed.run with N ranks on this node (one per GPU, rendezvous on
-    127.0.0.1), exactly as the driver launches it; rank 0 prints the line."""
+    torch.distributed.run with N ranks, exactly as the driver launches it; rank
+    0 prints the line."""
     import socket
     sock = socket.socket()
     sock.bind(("127.0.0.1", 0))
     port = sock.getsockname()[1]
     sock.close()
-    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
-           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
-    return subprocess.call(cmd)
+    return subprocess.call(relaunch_cmd(nproc, sys.argv[1:], port))
 
 
 def dist_env():
