@@ -42,6 +42,7 @@ struct Plan {
   size_t n = 0;
   uint64_t E_max = 0, chunks_max = 0;
   // workspace byte offsets
+  size_t o_scc = 0, o_idx = 0, o_ncnt = 0;   // zero-scalar compaction (non-prepared calls)
   size_t o_pts = 0, o_codes = 0, o_counts = 0, o_offsets = 0, o_cursor = 0, o_tiles = 0, o_vals = 0,
          o_spay = 0, o_heavy = 0, o_hlist = 0, o_hjobs = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_terms = 0, o_hot = 0, o_cb = 0, o_mcnt = 0, o_win = 0, total = 0;
   size_t seg_stride = 0;  // points between segT and segR in o_seg
@@ -282,6 +283,11 @@ struct Impl {
     size_t o = 0;
     auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
     p.o_pts = prepared ? 0 : take(n * 2 * N * 4);
+    if (!prepared) {
+      p.o_scc = take(n * NS * 4);
+      p.o_idx = take(n * 4);
+      p.o_ncnt = take(4);
+    }
     p.o_codes = take((size_t)p.W * n * 4);
     p.o_counts = take((size_t)p.M * 4);
     p.o_hot = take(((size_t)p.M + 31) / 32 * 4);
@@ -371,18 +377,20 @@ struct Impl {
   // a2 + a3: signed-window digits of every (point, window), bucket
   // histogram, exclusive scan -> offsets[0..M] (offsets[M] = E), and the
   // scatter of (point index | sign) into bucket order -> vals[0..E).
-  static gzkp_status sort_stage(const MsmCall& call, const Plan& p, char* ws, int* launches) {
+  static gzkp_status sort_stage(const MsmCall& call, const Plan& p, char* ws, int* launches,
+                                const uint32_t* scalars = nullptr, const uint32_t* n_live = nullptr) {
     cudaStream_t s = call.stream;
     const size_t n = call.n;
     auto U = [&](size_t off) { return (uint32_t*)(ws + off); };
+    if (!scalars) scalars = (const uint32_t*)call.scalars;
     // a2: digits + histogram
     GZ_CHECK(cudaMemsetAsync(U(p.o_counts), 0, (size_t)p.M * 4, s));
     GZ_CHECK(cudaMemsetAsync(U(p.o_hot), 0, ((size_t)p.M + 31) / 32 * 4, s));
     GZ_CHECK(cudaMemsetAsync(U(p.o_mcnt), 0, 4 * (p.groups.size() + 1), s));
     GZ_CHECK(cudaMemsetAsync(U(p.o_heavy), 0, 4 * (p.groups.size() + 4), s));
     const uint32_t bpw = (uint32_t)((n + DIGIT_THREADS - 1) / DIGIT_THREADS);
-    k_digits<C><<<bpw, DIGIT_THREADS, 0, s>>>((const uint32_t*)call.scalars, n, p.c, p.W, p.B, (uint32_t)p.Mi, U(p.o_codes),
-                                              U(p.o_counts));
+    k_digits<C><<<bpw, DIGIT_THREADS, 0, s>>>(scalars, n, p.c, p.W, p.B, (uint32_t)p.Mi, U(p.o_codes),
+                                              U(p.o_counts), n_live);
     GZ_CHECK(cudaGetLastError());
     // exclusive scan -> offsets (+ cursor copy); offsets[M] = E
     const uint32_t ntiles = (uint32_t)((p.M + SCAN_TILE - 1) / SCAN_TILE);
@@ -392,7 +400,8 @@ struct Impl {
     // a3: scatter into bucket order (window-major grid)
     const uint32_t bpw_s = (uint32_t)((n + SCATTER_TILE - 1) / SCATTER_TILE);
     k_scatter<<<(unsigned)((uint64_t)bpw_s * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw_s, p.B, (uint32_t)p.Mi,
-                                                                         p.val_stride, U(p.o_hot), U(p.o_cursor), U(p.o_vals));
+                                                                         p.val_stride, U(p.o_hot), U(p.o_cursor), U(p.o_vals),
+                                                                         n_live);
     GZ_CHECK(cudaGetLastError());
     *launches += 5;
     return GZKP_SUCCESS;
@@ -484,13 +493,23 @@ struct Impl {
 
     // a1: points -> Montgomery (skipped for prepared handles)
     const uint32_t* pts = (const uint32_t*)call.points;
+    const uint32_t* sc_sorted = nullptr;
+    const uint32_t* n_live = nullptr;
     if (!call.prepared) {
-      if (gzkp_status st = to_mont_sc(call.points, U(p.o_pts), n, call.scalars, s)) return st;
+      // drop the zero scalars, then convert the remaining points (compacted order)
+      GZ_CHECK(cudaMemsetAsync(U(p.o_ncnt), 0, 4, s));
+      k_compact<C><<<(unsigned)((n + 255) / 256), 256, 0, s>>>((const uint32_t*)call.scalars, n, U(p.o_scc), U(p.o_idx),
+                                                              U(p.o_ncnt));
+      const int cgrid = (int)std::min<size_t>((n + 255) / 256, (size_t)sms * 16);
+      k_to_mont_c<C><<<cgrid, 256, 0, s>>>((const uint32_t*)call.points, U(p.o_idx), U(p.o_ncnt), U(p.o_pts));
+      GZ_CHECK(cudaGetLastError());
       pts = U(p.o_pts);
-      ++launches;
+      sc_sorted = U(p.o_scc);
+      n_live = U(p.o_ncnt);
+      launches += 2;
     }
     // a2 + a3: signed digits, bucket histogram, offsets, sort by bucket
-    if (gzkp_status st = sort_stage(call, p, ws, &launches)) return st;
+    if (gzkp_status st = sort_stage(call, p, ws, &launches, sc_sorted, n_live)) return st;
     cudaEvent_t ev_sorted = profile_event(prof, s);
     profile_interval(prof, 0, ev_begin, ev_sorted);
 

@@ -93,6 +93,84 @@ __global__ void __launch_bounds__(256) k_to_mont(const uint32_t* __restrict__ in
   }
 }
 
+// ------------------------------------------- zero-scalar compaction (a1)
+// A zero scalar contributes nothing (half of the sparse
+// witness's scalars are 0).  k_compact keeps the points with a non-zero
+// scalar: their scalars go to sc_c and their indices to idx (block-level
+// ballot scan, one atomic per block), so the digit codes, the sort and the
+// point conversion only see the n' <= n live points (n' in *count).  The
+// order of the blocks is unspecified; the sum does not depend on it.  A bucket
+// entry then names the compacted point j; k_to_mont_c writes the Montgomery
+// form of point idx[j] to pts_c[j], full warps (no idle lanes on zero scalars).
+template <class C>
+__global__ void __launch_bounds__(256) k_compact(const uint32_t* __restrict__ sc, size_t n, uint32_t* __restrict__ sc_c,
+                                                 uint32_t* __restrict__ idx, uint32_t* __restrict__ count) {
+  constexpr int NS = C::NS;
+  __shared__ uint32_t s_warp[8], s_base;
+  const size_t i = (size_t)blockIdx.x * 256 + threadIdx.x;
+  uint32_t k[NS];
+  bool nz = false;
+  if (i < n) {
+    if constexpr (NS % 4 == 0) {
+      const uint4* src = reinterpret_cast<const uint4*>(sc + i * NS);
+#pragma unroll
+      for (int q = 0; q < NS / 4; ++q) {
+        const uint4 v = __ldg(src + q);
+        k[4 * q] = v.x; k[4 * q + 1] = v.y; k[4 * q + 2] = v.z; k[4 * q + 3] = v.w;
+      }
+    } else {
+#pragma unroll
+      for (int q = 0; q < NS; ++q) k[q] = __ldg(sc + i * NS + q);
+    }
+    uint32_t any = 0;
+#pragma unroll
+    for (int q = 0; q < NS; ++q) any |= k[q];
+    nz = any != 0;
+  }
+  const unsigned m = __ballot_sync(0xffffffffu, nz);
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  if (lane == 0) s_warp[w] = __popc(m);
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    uint32_t tot = 0;
+#pragma unroll
+    for (int q = 0; q < 8; ++q) { const uint32_t c = s_warp[q]; s_warp[q] = tot; tot += c; }
+    s_base = tot ? atomicAdd(count, tot) : 0u;
+  }
+  __syncthreads();
+  if (nz) {
+    const uint32_t pos = s_base + s_warp[w] + __popc(m & ((1u << lane) - 1u));
+    if constexpr (NS % 4 == 0) {
+      uint4* dst = reinterpret_cast<uint4*>(sc_c + (size_t)pos * NS);
+#pragma unroll
+      for (int q = 0; q < NS / 4; ++q) dst[q] = make_uint4(k[4 * q], k[4 * q + 1], k[4 * q + 2], k[4 * q + 3]);
+    } else {
+#pragma unroll
+      for (int q = 0; q < NS; ++q) sc_c[(size_t)pos * NS + q] = k[q];
+    }
+    idx[pos] = (uint32_t)i;
+  }
+}
+
+template <class C>
+__global__ void __launch_bounds__(256) k_to_mont_c(const uint32_t* __restrict__ in, const uint32_t* __restrict__ idx,
+                                                   const uint32_t* __restrict__ count, uint32_t* __restrict__ out) {
+  using Fp = Field<C>;
+  using E = EC<C>;
+  constexpr int N = C::N;
+  const uint32_t n = *count;
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
+    const size_t i = __ldg(idx + j);
+    uint32_t x[N], y[N];
+    E::ld(x, in + i * 2 * N);
+    E::ld(y, in + i * 2 * N + N);
+    Fp::to_mont(x, x);
+    Fp::to_mont(y, y);
+    E::st(out + (size_t)j * 2 * N, x);
+    E::st(out + (size_t)j * 2 * N + N, y);
+  }
+}
+
 // ------------------------------------------ block-level hot-key aggregation
 // Skewed scalars (the sparse witness: 40 % of the scalars are 1)
 // send one bucket a large share of all entries.  Warp aggregation leaves one
@@ -134,13 +212,18 @@ constexpr int DIG_SMALL_WIN = 64;             // small table: W <= 64 windows
 template <class C>
 __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __restrict__ sc, size_t n, int c, int W,
                                                           uint32_t B, uint32_t Mi, uint32_t* __restrict__ codes,
-                                                          uint32_t* __restrict__ counts) {
+                                                          uint32_t* __restrict__ counts,
+                                                          const uint32_t* __restrict__ n_live) {
+  // n: the codes' row stride; n_live (device, may be null): the points that
+  // exist (the compacted count), n_live <= n
   constexpr int NS = C::NS;
   __shared__ uint32_t s_sc[NS * DIGIT_THREADS];
   __shared__ uint32_t s_key[HOT_SLOTS], s_cnt[HOT_SLOTS];
   __shared__ uint32_t s_small[DIG_SMALL_WIN * DIG_SMALL];
   const size_t base = (size_t)blockIdx.x * DIGIT_THREADS;
-  const size_t left = n > base ? n - base : 0;
+  const size_t nl = n_live ? (size_t)*n_live : n;
+  if (base >= nl) return;
+  const size_t left = nl - base;
   const int rows = left < (size_t)DIGIT_THREADS ? (int)left : DIGIT_THREADS;
   const bool use_small = W <= DIG_SMALL_WIN;
   if (threadIdx.x < HOT_SLOTS) { s_key[threadIdx.x] = HOT_EMPTY; s_cnt[threadIdx.x] = 0; }
@@ -217,9 +300,12 @@ constexpr uint32_t HOT_COUNT = 1024;
 static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32_t* __restrict__ codes, size_t n,
                                                              uint32_t bpw, uint32_t B, uint32_t Mi, uint32_t val_stride,
                                                              const uint32_t* __restrict__ hotbits,
-                                                             uint32_t* __restrict__ cursor, uint32_t* __restrict__ vals) {
+                                                             uint32_t* __restrict__ cursor, uint32_t* __restrict__ vals,
+                                                             const uint32_t* __restrict__ n_live) {
   __shared__ uint32_t s_key[HOT_SLOTS], s_cnt[HOT_SLOTS], s_base[HOT_SLOTS];
   const int tid = threadIdx.x;
+  const size_t nl = n_live ? (size_t)*n_live : n;              // codes exist for i < nl (row stride n)
+  if ((size_t)(blockIdx.x % bpw) * SCATTER_TILE >= nl) return;  // whole block past the live points
   if (tid < HOT_SLOTS) { s_key[tid] = HOT_EMPTY; s_cnt[tid] = 0; }
   __syncthreads();
   const uint32_t t = blockIdx.x / bpw;
@@ -227,12 +313,12 @@ static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32
   const size_t i0 = (size_t)(blockIdx.x % bpw) * SCATTER_TILE + (size_t)tid * SCATTER_PER_THREAD;
   const uint32_t* crow = codes + (size_t)t * n;
   uint32_t code[SCATTER_PER_THREAD];
-  if (i0 + SCATTER_PER_THREAD <= n && (n % 4) == 0) {
+  if (i0 + SCATTER_PER_THREAD <= nl && (n % 4) == 0) {
     const uint4 v = *reinterpret_cast<const uint4*>(crow + i0);
     code[0] = v.x; code[1] = v.y; code[2] = v.z; code[3] = v.w;
   } else {
 #pragma unroll
-    for (int q = 0; q < SCATTER_PER_THREAD; ++q) code[q] = i0 + q < n ? crow[i0 + q] : 0u;
+    for (int q = 0; q < SCATTER_PER_THREAD; ++q) code[q] = i0 + q < nl ? crow[i0 + q] : 0u;
   }
   const int lane = tid & 31;
   unsigned peers[SCATTER_PER_THREAD];
