@@ -286,7 +286,7 @@ struct Impl {
     if (!prepared) {
       p.o_scc = take(n * NS * 4);
       p.o_idx = take(n * 4);
-      p.o_ncnt = take(4);
+      p.o_ncnt = take(4 * 8);      // counters [2] + ranges [4]
     }
     p.o_codes = take((size_t)p.W * n * 4);
     p.o_counts = take((size_t)p.M * 4);
@@ -378,7 +378,7 @@ struct Impl {
   // histogram, exclusive scan -> offsets[0..M] (offsets[M] = E), and the
   // scatter of (point index | sign) into bucket order -> vals[0..E).
   static gzkp_status sort_stage(const MsmCall& call, const Plan& p, char* ws, int* launches,
-                                const uint32_t* scalars = nullptr, const uint32_t* n_live = nullptr) {
+                                const uint32_t* scalars = nullptr, const uint32_t* rng = nullptr) {
     cudaStream_t s = call.stream;
     const size_t n = call.n;
     auto U = [&](size_t off) { return (uint32_t*)(ws + off); };
@@ -389,8 +389,13 @@ struct Impl {
     GZ_CHECK(cudaMemsetAsync(U(p.o_mcnt), 0, 4 * (p.groups.size() + 1), s));
     GZ_CHECK(cudaMemsetAsync(U(p.o_heavy), 0, 4 * (p.groups.size() + 4), s));
     const uint32_t bpw = (uint32_t)((n + DIGIT_THREADS - 1) / DIGIT_THREADS);
+    // rng (compaction): big range [rng[0], rng[1]) every window, small range
+    // [rng[2], rng[3]) window 0 only; grids sized for n, blocks past a range exit
     k_digits<C><<<bpw, DIGIT_THREADS, 0, s>>>(scalars, n, p.c, p.W, p.B, (uint32_t)p.Mi, U(p.o_codes),
-                                              U(p.o_counts), n_live);
+                                              U(p.o_counts), rng);
+    if (rng)
+      k_digits<C><<<bpw, DIGIT_THREADS, 0, s>>>(scalars, n, p.c, 1, p.B, (uint32_t)p.Mi, U(p.o_codes),
+                                                U(p.o_counts), rng + 2);
     GZ_CHECK(cudaGetLastError());
     // exclusive scan -> offsets (+ cursor copy); offsets[M] = E
     const uint32_t ntiles = (uint32_t)((p.M + SCAN_TILE - 1) / SCAN_TILE);
@@ -401,7 +406,10 @@ struct Impl {
     const uint32_t bpw_s = (uint32_t)((n + SCATTER_TILE - 1) / SCATTER_TILE);
     k_scatter<<<(unsigned)((uint64_t)bpw_s * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw_s, p.B, (uint32_t)p.Mi,
                                                                          p.val_stride, U(p.o_hot), U(p.o_cursor), U(p.o_vals),
-                                                                         n_live);
+                                                                         rng);
+    if (rng)
+      k_scatter<<<bpw_s, SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw_s, p.B, (uint32_t)p.Mi, p.val_stride, U(p.o_hot),
+                                                  U(p.o_cursor), U(p.o_vals), rng + 2);
     GZ_CHECK(cudaGetLastError());
     *launches += 5;
     return GZKP_SUCCESS;
@@ -494,22 +502,24 @@ struct Impl {
     // a1: points -> Montgomery (skipped for prepared handles)
     const uint32_t* pts = (const uint32_t*)call.points;
     const uint32_t* sc_sorted = nullptr;
-    const uint32_t* n_live = nullptr;
+    const uint32_t* rng = nullptr;
     if (!call.prepared) {
-      // drop the zero scalars, then convert the remaining points (compacted order)
-      GZ_CHECK(cudaMemsetAsync(U(p.o_ncnt), 0, 4, s));
-      k_compact<C><<<(unsigned)((n + 255) / 256), 256, 0, s>>>((const uint32_t*)call.scalars, n, U(p.o_scc), U(p.o_idx),
-                                                              U(p.o_ncnt));
+      // drop the zero scalars (small ones to the back), then convert the
+      // remaining points in the compacted order
+      GZ_CHECK(cudaMemsetAsync(U(p.o_ncnt), 0, 8, s));
+      k_compact<C><<<(unsigned)((n + 255) / 256), 256, 0, s>>>((const uint32_t*)call.scalars, n, p.c, U(p.o_scc),
+                                                              U(p.o_idx), U(p.o_ncnt));
+      k_compact_ranges<<<1, 1, 0, s>>>(U(p.o_ncnt), (uint32_t)n, U(p.o_ncnt) + 2);
       const int cgrid = (int)std::min<size_t>((n + 255) / 256, (size_t)sms * 16);
-      k_to_mont_c<C><<<cgrid, 256, 0, s>>>((const uint32_t*)call.points, U(p.o_idx), U(p.o_ncnt), U(p.o_pts));
+      k_to_mont_c<C><<<cgrid, 256, 0, s>>>((const uint32_t*)call.points, U(p.o_idx), U(p.o_ncnt) + 2, U(p.o_pts));
       GZ_CHECK(cudaGetLastError());
       pts = U(p.o_pts);
       sc_sorted = U(p.o_scc);
-      n_live = U(p.o_ncnt);
-      launches += 2;
+      rng = U(p.o_ncnt) + 2;
+      launches += 5;
     }
     // a2 + a3: signed digits, bucket histogram, offsets, sort by bucket
-    if (gzkp_status st = sort_stage(call, p, ws, &launches, sc_sorted, n_live)) return st;
+    if (gzkp_status st = sort_stage(call, p, ws, &launches, sc_sorted, rng)) return st;
     cudaEvent_t ev_sorted = profile_event(prof, s);
     profile_interval(prof, 0, ev_begin, ev_sorted);
 

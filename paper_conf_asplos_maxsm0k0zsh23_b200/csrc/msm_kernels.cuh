@@ -102,14 +102,20 @@ __global__ void __launch_bounds__(256) k_to_mont(const uint32_t* __restrict__ in
 // order of the blocks is unspecified; the sum does not depend on it.  A bucket
 // entry then names the compacted point j; k_to_mont_c writes the Montgomery
 // form of point idx[j] to pts_c[j], full warps (no idle lanes on zero scalars).
+// Scalars below 2^(c-1) ("small": the 1s of the sparse witness) have one
+// non-zero signed digit, in window 0, so they are packed at the END of the
+// compacted arrays, [n - n_small, n), and the digit and scatter kernels run
+// every window over the "big" range [0, n_big) but only window 0 over the
+// small range.  count[0] = n_big, count[1] = n_small.
 template <class C>
-__global__ void __launch_bounds__(256) k_compact(const uint32_t* __restrict__ sc, size_t n, uint32_t* __restrict__ sc_c,
-                                                 uint32_t* __restrict__ idx, uint32_t* __restrict__ count) {
+__global__ void __launch_bounds__(256) k_compact(const uint32_t* __restrict__ sc, size_t n, int c,
+                                                 uint32_t* __restrict__ sc_c, uint32_t* __restrict__ idx,
+                                                 uint32_t* __restrict__ count) {
   constexpr int NS = C::NS;
-  __shared__ uint32_t s_warp[8], s_base;
+  __shared__ uint32_t s_warp[8], s_wsm[8], s_base, s_sbase;
   const size_t i = (size_t)blockIdx.x * 256 + threadIdx.x;
   uint32_t k[NS];
-  bool nz = false;
+  bool nz = false, small = false;
   if (i < n) {
     if constexpr (NS % 4 == 0) {
       const uint4* src = reinterpret_cast<const uint4*>(sc + i * NS);
@@ -122,24 +128,34 @@ __global__ void __launch_bounds__(256) k_compact(const uint32_t* __restrict__ sc
 #pragma unroll
       for (int q = 0; q < NS; ++q) k[q] = __ldg(sc + i * NS + q);
     }
-    uint32_t any = 0;
+    uint32_t any = 0, high = 0;
 #pragma unroll
     for (int q = 0; q < NS; ++q) any |= k[q];
+#pragma unroll
+    for (int q = 1; q < NS; ++q) high |= k[q];
     nz = any != 0;
+    small = nz && high == 0 && k[0] < (1u << (c - 1));
   }
-  const unsigned m = __ballot_sync(0xffffffffu, nz);
+  const bool big = nz && !small;
+  const unsigned m = __ballot_sync(0xffffffffu, big), ms = __ballot_sync(0xffffffffu, small);
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  if (lane == 0) s_warp[w] = __popc(m);
+  if (lane == 0) { s_warp[w] = __popc(m); s_wsm[w] = __popc(ms); }
   __syncthreads();
   if (threadIdx.x == 0) {
-    uint32_t tot = 0;
+    uint32_t tot = 0, tots = 0;
 #pragma unroll
-    for (int q = 0; q < 8; ++q) { const uint32_t c = s_warp[q]; s_warp[q] = tot; tot += c; }
+    for (int q = 0; q < 8; ++q) {
+      const uint32_t cb = s_warp[q], cs = s_wsm[q];
+      s_warp[q] = tot; tot += cb;
+      s_wsm[q] = tots; tots += cs;
+    }
     s_base = tot ? atomicAdd(count, tot) : 0u;
+    s_sbase = tots ? atomicAdd(count + 1, tots) : 0u;
   }
   __syncthreads();
   if (nz) {
-    const uint32_t pos = s_base + s_warp[w] + __popc(m & ((1u << lane) - 1u));
+    const uint32_t pos = big ? s_base + s_warp[w] + __popc(m & ((1u << lane) - 1u))
+                             : (uint32_t)(n - 1 - (s_sbase + s_wsm[w] + __popc(ms & ((1u << lane) - 1u))));
     if constexpr (NS % 4 == 0) {
       uint4* dst = reinterpret_cast<uint4*>(sc_c + (size_t)pos * NS);
 #pragma unroll
@@ -152,14 +168,23 @@ __global__ void __launch_bounds__(256) k_compact(const uint32_t* __restrict__ sc
   }
 }
 
+// rng = {0, n_big, n - n_small, n}: the big and the small ranges
+static __global__ void k_compact_ranges(const uint32_t* __restrict__ count, uint32_t n, uint32_t* __restrict__ rng) {
+  rng[0] = 0;
+  rng[1] = count[0];
+  rng[2] = n - count[1];
+  rng[3] = n;
+}
+
 template <class C>
 __global__ void __launch_bounds__(256) k_to_mont_c(const uint32_t* __restrict__ in, const uint32_t* __restrict__ idx,
-                                                   const uint32_t* __restrict__ count, uint32_t* __restrict__ out) {
+                                                   const uint32_t* __restrict__ rng, uint32_t* __restrict__ out) {
   using Fp = Field<C>;
   using E = EC<C>;
   constexpr int N = C::N;
-  const uint32_t n = *count;
-  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
+  const uint32_t nb = rng[1], s0 = rng[2], n = nb + (rng[3] - s0);
+  for (uint32_t v = blockIdx.x * blockDim.x + threadIdx.x; v < n; v += gridDim.x * blockDim.x) {
+    const uint32_t j = v < nb ? v : s0 + (v - nb);
     const size_t i = __ldg(idx + j);
     uint32_t x[N], y[N];
     E::ld(x, in + i * 2 * N);
@@ -213,17 +238,18 @@ template <class C>
 __global__ void __launch_bounds__(DIGIT_THREADS) k_digits(const uint32_t* __restrict__ sc, size_t n, int c, int W,
                                                           uint32_t B, uint32_t Mi, uint32_t* __restrict__ codes,
                                                           uint32_t* __restrict__ counts,
-                                                          const uint32_t* __restrict__ n_live) {
-  // n: the codes' row stride; n_live (device, may be null): the points that
-  // exist (the compacted count), n_live <= n
+                                                          const uint32_t* __restrict__ rng) {
+  // n: the codes' row stride; rng (device, may be null = [0, n)): the point
+  // range [rng[0], rng[1]) this launch covers; W: the windows it writes (1
+  // for the small-scalar range of the compaction)
   constexpr int NS = C::NS;
   __shared__ uint32_t s_sc[NS * DIGIT_THREADS];
   __shared__ uint32_t s_key[HOT_SLOTS], s_cnt[HOT_SLOTS];
   __shared__ uint32_t s_small[DIG_SMALL_WIN * DIG_SMALL];
-  const size_t base = (size_t)blockIdx.x * DIGIT_THREADS;
-  const size_t nl = n_live ? (size_t)*n_live : n;
-  if (base >= nl) return;
-  const size_t left = nl - base;
+  const size_t lo = rng ? (size_t)rng[0] : 0, hi = rng ? (size_t)rng[1] : n;
+  const size_t base = lo + (size_t)blockIdx.x * DIGIT_THREADS;
+  if (base >= hi) return;
+  const size_t left = hi - base;
   const int rows = left < (size_t)DIGIT_THREADS ? (int)left : DIGIT_THREADS;
   const bool use_small = W <= DIG_SMALL_WIN;
   if (threadIdx.x < HOT_SLOTS) { s_key[threadIdx.x] = HOT_EMPTY; s_cnt[threadIdx.x] = 0; }
@@ -301,24 +327,25 @@ static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32
                                                              uint32_t bpw, uint32_t B, uint32_t Mi, uint32_t val_stride,
                                                              const uint32_t* __restrict__ hotbits,
                                                              uint32_t* __restrict__ cursor, uint32_t* __restrict__ vals,
-                                                             const uint32_t* __restrict__ n_live) {
+                                                             const uint32_t* __restrict__ rng) {
+  // codes exist for i in [lo, hi) (rng, device; null = [0, n)), row stride n
   __shared__ uint32_t s_key[HOT_SLOTS], s_cnt[HOT_SLOTS], s_base[HOT_SLOTS];
   const int tid = threadIdx.x;
-  const size_t nl = n_live ? (size_t)*n_live : n;              // codes exist for i < nl (row stride n)
-  if ((size_t)(blockIdx.x % bpw) * SCATTER_TILE >= nl) return;  // whole block past the live points
+  const size_t lo = rng ? (size_t)rng[0] : 0, hi = rng ? (size_t)rng[1] : n;
+  if (lo + (size_t)(blockIdx.x % bpw) * SCATTER_TILE >= hi) return;   // whole block past the range
   if (tid < HOT_SLOTS) { s_key[tid] = HOT_EMPTY; s_cnt[tid] = 0; }
   __syncthreads();
   const uint32_t t = blockIdx.x / bpw;
   const uint32_t kbase = t % Mi * B, vbase = t / Mi * val_stride;
-  const size_t i0 = (size_t)(blockIdx.x % bpw) * SCATTER_TILE + (size_t)tid * SCATTER_PER_THREAD;
+  const size_t i0 = lo + (size_t)(blockIdx.x % bpw) * SCATTER_TILE + (size_t)tid * SCATTER_PER_THREAD;
   const uint32_t* crow = codes + (size_t)t * n;
   uint32_t code[SCATTER_PER_THREAD];
-  if (i0 + SCATTER_PER_THREAD <= nl && (n % 4) == 0) {
+  if (i0 + SCATTER_PER_THREAD <= hi && (n % 4) == 0 && (i0 & 3) == 0) {
     const uint4 v = *reinterpret_cast<const uint4*>(crow + i0);
     code[0] = v.x; code[1] = v.y; code[2] = v.z; code[3] = v.w;
   } else {
 #pragma unroll
-    for (int q = 0; q < SCATTER_PER_THREAD; ++q) code[q] = i0 + q < nl ? crow[i0 + q] : 0u;
+    for (int q = 0; q < SCATTER_PER_THREAD; ++q) code[q] = i0 + q < hi ? crow[i0 + q] : 0u;
   }
   const int lane = tid & 31;
   unsigned peers[SCATTER_PER_THREAD];
