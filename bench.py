@@ -291,7 +291,7 @@ def run_ntt(args, wl):
     world, rank, local = dist_env()
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dist.init_process_group("gloo")   # host plumbing only: barriers, max over ranks
     if not os.path.exists(gz.LIB_PATH) and rank == 0:
         gbuild.build()
     if world > 1:
@@ -326,7 +326,7 @@ def run_ntt(args, wl):
         torch.cuda.synchronize()
         total_ms += e0.elapsed_time(e1)
     clocks = sampler.stop()
-    t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+    t = torch.tensor([total_ms], dtype=torch.float64)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     ms = float(t.item()) / args.steps
@@ -412,8 +412,10 @@ def main():
     if "WORLD_SIZE" in os.environ and int(os.environ["WORLD_SIZE"]) != args.gpus:
         sys.exit(f"bench.py: WORLD_SIZE={os.environ['WORLD_SIZE']} but --gpus {args.gpus}")
     if int(os.environ.get("WORLD_SIZE", "1")) > 1:
-        # the communicator set-up log (one "comm ... rank r nranks N" line per
-        # rank) shows which ranks and transports the collective really used
+        # the communicator set-up log of the MSM's NCCL communicator (one
+        # "comm ... rank r nranks N" line per rank) shows which ranks and
+        # transports the all-gather really used; torch's own process group is
+        # gloo (host plumbing only), so this is the only NCCL communicator
         os.environ.setdefault("NCCL_DEBUG", "INFO")
         os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
 
@@ -436,7 +438,7 @@ def main():
     world, rank, local = dist_env()
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dist.init_process_group("gloo")   # host plumbing only: barriers, max over ranks
     # the in-tree libgzkp.so travels with the repo; only a missing library is
     # built, by rank 0 alone (never N concurrent nvcc runs)
     if not os.path.exists(gz.LIB_PATH) and rank == 0:
@@ -529,7 +531,7 @@ def main():
     gz.set_profiling(False)
     result = gz.to_numpy(out).copy()          # the timed steps' MSM value (parity leg below)
 
-    t = torch.tensor([total_ms], dtype=torch.float64, device="cuda")
+    t = torch.tensor([total_ms], dtype=torch.float64)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     total_ms = float(t.item())
@@ -570,7 +572,7 @@ def main():
         pprof = gz.profile_read(reset=True)
         gz.set_profiling(False)
         presult = gz.to_numpy(pout).copy()
-        tp = torch.tensor([pe0.elapsed_time(pe1)], dtype=torch.float64, device="cuda")
+        tp = torch.tensor([pe0.elapsed_time(pe1)], dtype=torch.float64)
         if world > 1:
             dist.all_reduce(tp, op=dist.ReduceOp.MAX)
         p_ms = float(tp.item()) / args.steps
@@ -659,7 +661,7 @@ def main():
                 outh.copy_(o, non_blocking=True)
                 torch.cuda.synchronize()
             e2e_ms = (time.perf_counter() - t0) * 1e3 / k_e2e
-            te = torch.tensor([e2e_ms], dtype=torch.float64, device="cuda")
+            te = torch.tensor([e2e_ms], dtype=torch.float64)
             dist.all_reduce(te, op=dist.ReduceOp.MAX)
             e2e_ms = float(te.item())
         e2e = {"value": n / (e2e_ms / 1e3), "unit": "points/s", "ms_per_step": e2e_ms,
