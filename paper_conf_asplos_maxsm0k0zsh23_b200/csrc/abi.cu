@@ -7,6 +7,7 @@
 #include <dlfcn.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cstdint>
 #include <cstdio>
 #include <cstdlib>
@@ -46,13 +47,16 @@ int device_sm_count() {
   return sms > 0 ? sms : 148;
 }
 
-static int g_profiling = -1;
+static std::atomic<int> g_profiling{-1};
 bool profiling_enabled() {
-  if (g_profiling < 0) {
+  int v = g_profiling.load(std::memory_order_relaxed);
+  if (v < 0) {
     const char* e = getenv("GZKP_PROFILE");
-    g_profiling = (e && atoi(e) != 0) ? 1 : 0;
+    int expect = -1;
+    g_profiling.compare_exchange_strong(expect, (e && atoi(e) != 0) ? 1 : 0);
+    v = g_profiling.load(std::memory_order_relaxed);
   }
-  return g_profiling == 1;
+  return v == 1;
 }
 
 // pending records of this thread, harvested by gzkp_profile_read
@@ -474,7 +478,7 @@ gzkp_status gzkp_msm_host(int curve, const void* points_host, const void* scalar
     call.out_affine = dout;
     call.stream = s;
     call.points_ready = n ? ev_points : nullptr;
-    st = n ? c->msm(call) : c->msm(call);
+    st = c->msm(call);
   }
   if (!st && (e = cudaMemcpyAsync(out_host, dout, ob, cudaMemcpyDeviceToHost, s)) != cudaSuccess) st = cuda_status(e, "D2H out");
   cudaStreamWaitEvent(s, ev_points, 0);   // never free while the side stream may still copy
@@ -631,7 +635,7 @@ gzkp_status gzkp_set_config(int window_bits, int chunk_entries) {
 }
 
 gzkp_status gzkp_set_profiling(int on) {
-  g_profiling = on ? 1 : 0;
+  g_profiling.store(on ? 1 : 0);
   return GZKP_SUCCESS;
 }
 
