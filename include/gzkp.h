@@ -124,7 +124,7 @@ gzkp_status gzkp_msm_host(int curve, const void *points_affine_host, const void 
  *   window_bits = 0 lets the planner choose c, else 2..22; later MSMs on the
  *   handle use that c.
  * weighted = 0: Montgomery-form copy of the points only (standard pipeline);
- *   window_bits 0 (planner per call) or 2..16 (fixed c for every call).
+ *   window_bits 0 (planner per call) or 2..18 (fixed c for every call).
  *   Other values: GZKP_ERROR_INVALID_VALUE.
  * gzkp_points_prepare = _ex(window_bits 0, weighted 1), falling back to
  * weighted 0 if the table does not fit.  gzkp_prepared_info reports the window
@@ -197,7 +197,7 @@ gzkp_status gzkp_fixed_base_mul(int curve, const void *scalars, size_t n, void *
 /* Test hook (not on the MSM path): runs ONLY the product's digit + sort stage
  * (a2-a3: signed c-bit windows, §2.3 / Figure 3; the bucket
  * layout p_index of PAPER.md:206) for `scalars` (device, n x scalar_bytes) at
- * window bits c in 2..16, synchronises, and copies to HOST memory:
+ * window bits c in 2..18, synchronises, and copies to HOST memory:
  *   offsets_host[0 .. W 2^(c-1)]: bucket key t 2^(c-1) + |d| - 1 (window t,
  *     digit d != 0) owns entries [offsets[key], offsets[key+1]);
  *   vals_host[0 .. E): point index | 0x80000000 if the digit is negative,
@@ -224,7 +224,7 @@ gzkp_status gzkp_field_op(int curve, int op, const void *a, const void *b, void 
  * 3: 2P via mdbl. */
 gzkp_status gzkp_ec_op(int curve, int op, const void *P, const void *Q, void *out, size_t n,
                        gzkp_stream stream);
-/* Tunables (0 = automatic): window bits c, entries per accumulation chunk. */
+/* Tunables (0 = automatic): window bits c (2..18), entries per accumulation chunk. */
 gzkp_status gzkp_set_config(int window_bits, int chunk_entries);
 /* Plan the window size the library would use for (curve, n). */
 int gzkp_window_bits(int curve, size_t n);

@@ -496,8 +496,8 @@ gzkp_status gzkp_points_prepare_ex(int curve, const void* points_affine, size_t 
     return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
   // the standard (per-window bucket sets) pipeline plans c <= 16, as gzkp_set_config
   if (weighted < 0) return set_error(GZKP_ERROR_INVALID_VALUE, "weighted (checkpoint interval) must be >= 0");
-  if (weighted == 0 && (window_bits == 1 || window_bits > 16))
-    return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..16 for unweighted points");
+  if (weighted == 0 && (window_bits == 1 || window_bits > 18))
+    return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..18 for unweighted points");
   if (weighted >= 1 && window_bits == 1) return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..22");
   if (gzkp_status st = debug_validate(c, points_affine, nullptr, n, (cudaStream_t)stream)) return st;
   Prepared* h = new (std::nothrow) Prepared{curve, n, nullptr, false, 0, 1, 0, 1};
@@ -627,8 +627,8 @@ gzkp_status gzkp_ec_op(int curve, int op, const void* P, const void* Q, void* ou
 }
 
 gzkp_status gzkp_set_config(int window_bits, int chunk_entries) {
-  if (window_bits < 0 || window_bits > 16 || window_bits == 1 || chunk_entries < 0 || chunk_entries > (1 << 20))
-    return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..16");
+  if (window_bits < 0 || window_bits > 18 || window_bits == 1 || chunk_entries < 0 || chunk_entries > (1 << 20))
+    return set_error(GZKP_ERROR_INVALID_VALUE, "window_bits must be 0 or 2..18");
   tunables().window_bits = window_bits;
   tunables().chunk_entries = chunk_entries;
   return GZKP_SUCCESS;
@@ -758,7 +758,7 @@ gzkp_status gzkp_debug_buckets(int curve, const void* scalars, size_t n, int win
                                size_t offsets_cap, uint32_t* vals_host, size_t vals_cap, gzkp_stream stream) {
   const CurveImpl* c = impl_for(curve);
   if (!c) return set_error(GZKP_ERROR_UNSUPPORTED_CURVE, "unknown curve");
-  if (window_bits < 2 || window_bits > 16 || !offsets_host || (n && (!scalars || !vals_host)) || !aligned16(scalars))
+  if (window_bits < 2 || window_bits > 18 || !offsets_host || (n && (!scalars || !vals_host)) || !aligned16(scalars))
     return set_error(GZKP_ERROR_INVALID_VALUE, "bad arguments");
   init_pool_once();
   return c->debug_buckets(scalars, n, window_bits, offsets_host, offsets_cap, vals_host, vals_cap,

@@ -70,13 +70,16 @@ struct Impl {
     if (tunables().window_bits > 0) return tunables().window_bits;
     if (const char* e = getenv("GZKP_WINDOW_BITS")) {
       int v = atoi(e);
-      if (v >= 2 && v <= 16) return v;
+      if (v >= 2 && v <= 18) return v;
     }
     const double madd = 10.0, add = 14.0, dbl = 10.0;
     const double lat = 6000.0;   // a serial op on one thread vs the whole chip's throughput
     int best = 8;
     double best_cost = 1e300;
-    const int cmax = C::SCALAR_BITS < 16 ? 4 : 16;
+    // c <= 18 (round 2, BLS12-381: 2^22 at c = 16 / 17 / 18 = 28.7 / 29.8 / 30.4 ms,
+    // 2^26 at c = 16 / 17 / 18 / 19 = 423.7 / 408.5 / 399.1 / 403.4 ms; the model
+    // keeps 16 up to 2^22 and takes 18 from 2^23 on)
+    const int cmax = C::SCALAR_BITS < 16 ? 4 : 18;
     for (int c = 2; c <= cmax; ++c) {
       const int W = (C::SCALAR_BITS + 1 + c - 1) / c;
       const double B = std::ldexp(1.0, c - 1);

@@ -69,7 +69,7 @@ def test_fig3_bucket_membership(curve):
 
 
 @pytest.mark.parametrize("curve,c", [("bn254", 2), ("bn254", 5), ("bn254", 16), ("bls12_381", 13),
-                                     ("bls12_381", 16), ("mnt4_753", 16), ("toy_a2", 3)])
+                                     ("bls12_381", 16), ("bls12_381", 18), ("mnt4_753", 16), ("toy_a2", 3)])
 @pytest.mark.parametrize("dist", ["uniform", "zcash_like", "r_minus_1", "full_bits", "small", "pow2"])
 def test_digits_reconstruct_scalars(curve, c, dist):
     gz = require_cuda()

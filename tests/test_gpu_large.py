@@ -111,7 +111,7 @@ def test_mnt4_window_invariance_at_bench_c(curve, dist):
     k = synth.scalars(curve, n, 33, dist)
     want = oracle.closed_form(curve, k, d)
     try:
-        for c in (4, 13, 16):
+        for c in (4, 13, 16, 18):
             for S in (1, 16, 64, 257):
                 gz.set_config(c, S)
                 assert np.array_equal(host(gz.msm(curve, dev(pts), dev(k))), want), (c, S)

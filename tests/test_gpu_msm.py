@@ -122,8 +122,8 @@ def test_invariance_window_and_chunk(curve):
     pts = pts[:n]
     k = synth.scalars(curve, n, 31, "zcash_like" if curve != "toy_a2" else "uniform")
     want = oracle_msm_cached(curve, pts, k)
-    cmax = 16 if curve != "toy_a2" else 4
-    for c in sorted({2, 3, 4, 7, 10, 13, cmax} & set(range(2, cmax + 1))):
+    cmax = 18 if curve != "toy_a2" else 4
+    for c in sorted({2, 3, 4, 7, 10, 13, 16, 17, cmax} & set(range(2, cmax + 1))):
         for S in (1, 3, 16, 64, 257):
             gz.set_config(c, S)
             got = run(gz, curve, pts, k)

@@ -51,4 +51,7 @@ def test_window_bits_planner_ranges():
     for curve in ("bn254", "bls12_381", "mnt4_753", "bn254_g2", "bls12_381_g2"):
         for logn in (0, 5, 10, 16, 19, 20, 22, 26):
             c = gz.window_bits(curve, 1 << logn)
-            assert 2 <= c <= 16, (curve, logn, c)
+            assert 2 <= c <= 18, (curve, logn, c)
+    # the benched configurations keep their measured window sizes
+    assert gz.window_bits("bls12_381", 1 << 22) == 16 and gz.window_bits("bls12_381", 1 << 26) == 18
+    assert gz.window_bits("bn254", 1 << 20) == 16 and gz.window_bits("mnt4_753", 1 << 20) == 16
