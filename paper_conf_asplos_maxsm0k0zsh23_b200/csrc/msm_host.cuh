@@ -76,10 +76,7 @@ struct Impl {
     const double lat = 6000.0;   // a serial op on one thread vs the whole chip's throughput
     int best = 8;
     double best_cost = 1e300;
-    // c <= 18 (round 2, BLS12-381: 2^22 at c = 16 / 17 / 18 = 28.7 / 29.8 / 30.4 ms,
-    // 2^26 at c = 16 / 17 / 18 / 19 = 423.7 / 408.5 / 399.1 / 403.4 ms; the model
-    // keeps 16 up to 2^22 and takes 18 from 2^23 on)
-    const int cmax = C::SCALAR_BITS < 16 ? 4 : 18;
+    const int cmax = C::SCALAR_BITS < 16 ? 4 : 16;
     for (int c = 2; c <= cmax; ++c) {
       const int W = (C::SCALAR_BITS + 1 + c - 1) / c;
       const double B = std::ldexp(1.0, c - 1);
@@ -91,6 +88,13 @@ struct Impl {
       const double cost = entries * madd + reduce + tail + top_window_merge(n, c, W) * add * lat;
       if (cost < best_cost) { best_cost = cost; best = c; }
     }
+    // Measured override for the ~255-bit scalar fields at n >= 2^24 (round 2,
+    // BLS12-381 2^26: uniform at c = 16 / 17 / 18 = 423.7 / 408.5 / 399.1 ms,
+    // the sparse witness 42.77 / 42.75 / 44.61 ms; 2^22 uniform 28.7 / 29.8 /
+    // 30.4 ms): c = 17 leaves the top window one bit wide, so ~15.5 windows
+    // carry entries instead of 16, which the model's n W entries miss; 18 is
+    // faster still on uniform scalars but slower on the sparse witness.
+    if (C::SCALAR_BITS >= 250 && C::SCALAR_BITS <= 256 && n >= (1ull << 24) && best == 16) best = 17;
     return best;
   }
 

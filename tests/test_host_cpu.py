@@ -53,5 +53,5 @@ def test_window_bits_planner_ranges():
             c = gz.window_bits(curve, 1 << logn)
             assert 2 <= c <= 18, (curve, logn, c)
     # the benched configurations keep their measured window sizes
-    assert gz.window_bits("bls12_381", 1 << 22) == 16 and gz.window_bits("bls12_381", 1 << 26) == 18
+    assert gz.window_bits("bls12_381", 1 << 22) == 16 and gz.window_bits("bls12_381", 1 << 26) == 17
     assert gz.window_bits("bn254", 1 << 20) == 16 and gz.window_bits("mnt4_753", 1 << 20) == 16
