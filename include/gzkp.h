@@ -45,9 +45,19 @@
  * GZKP_ERROR_INVALID_VALUE (detail in gzkp_last_error) before any MSM work.
  * No exception crosses the ABI; gzkp_last_error() gives thread-local detail.
  *
- * THREADING: calls on different streams are independent (each call owns its
- * workspace).  Two concurrent gzkp_msm_sharded calls on one communicator are
- * not allowed (NCCL ordering rule).
+ * THREADING: calls on different streams are independent: the library keeps
+ * one workspace and one pair of side streams per (device, stream) -- per
+ * (device, stream, thread) for cudaStreamPerThread -- and calls on one stream
+ * are ordered by it.  Per-device setup (kernel attributes, the private memory
+ * pool, the stack limit) runs once per device, so one process may drive
+ * several GPUs.  Release a stream's resources with gzkp_release_stream before
+ * destroying it.  Two concurrent gzkp_msm_sharded calls on one communicator
+ * are not allowed (NCCL ordering rule).
+ *
+ * WORK SKIPPED BY DEFINITION: a zero scalar contributes nothing; gzkp_msm /
+ * _ex / _partial drop those points before the sort (and convert only the rest
+ * to Montgomery form), so sparse scalar vectors cost in
+ * proportion to their non-zero entries.
  */
 #ifndef GZKP_H
 #define GZKP_H
