@@ -53,8 +53,13 @@ struct Plan {
     int heavy_levels;
     uint32_t hmax, hbase;       // heavy-list capacity and first entry
     int seg = 16;               // reduction segment (buckets per thread)
+    // reduction sub-groups, top windows first: the Horner tail of sub-group k
+    // (side stream 2) overlaps the reduction of sub-group k+1 (GZKP_REDUCE_GROUPS)
+    struct Sub { int t_lo, t_hi, seg; };
+    std::vector<Sub> subs;
   };
   std::vector<Grp> groups;
+  bool split_reduce = false;    // more than one reduction sub-group somewhere: side streams needed
 };
 
 inline int ilog2_u64(uint64_t v) { int r = 0; while (v > 1) { v >>= 1; ++r; } return r; }
@@ -267,14 +272,38 @@ struct Impl {
         const long v = e ? atol(e) : 32768;
         return (uint64_t)(v > 0 ? v : 32768);
       }();
-      uint64_t seg = 16;
-      while (seg > 1 && bwins * p.B / seg < target) seg >>= 1;
-      g.seg = (int)std::min<uint64_t>(seg, p.B);
-      const uint64_t gsegs = p.B / g.seg;
-      seg_elems = std::max<uint64_t>(seg_elems, bwins * gsegs);
-      const uint64_t nb_bits = (uint64_t)ilog2_u64(gsegs) + 1;           // NB + 1 sets
-      mid_elems = std::max<uint64_t>(mid_elems, bwins * nb_bits * ((gsegs + RB_PER - 1) / RB_PER));
-      terms_elems = std::max<uint64_t>(terms_elems, bwins * nb_bits);
+      auto seg_for = [&](uint64_t w) {
+        uint64_t sg = 16;
+        while (sg > 1 && w * p.B / sg < target) sg >>= 1;
+        return (int)std::min<uint64_t>(sg, p.B);
+      };
+      g.seg = seg_for(bwins);
+      // sub-groups: consolidated tables keep one (their M bucket sets are short)
+      static const int rgroups = [] {
+        const char* e = getenv("GZKP_REDUCE_GROUPS");
+        const int v = e ? atoi(e) : 1;
+        return v >= 1 ? v : 1;
+      }();
+      g.subs.clear();
+      const int R = consolidated ? 1 : std::max(1, std::min<int>(rgroups, (int)wins));
+      {
+        int hi = consolidated ? p.Mi - 1 : g.t_hi;
+        const int lo_all = consolidated ? 0 : g.t_lo;
+        for (int k = 0; k < R; ++k) {
+          const int rem = hi - lo_all + 1, sz = (rem + (R - k) - 1) / (R - k);
+          g.subs.push_back({hi - sz + 1, hi, seg_for((uint64_t)sz)});
+          hi -= sz;
+        }
+      }
+      if (R > 1) p.split_reduce = true;
+      for (const auto& sb : g.subs) {
+        const uint64_t sw = (uint64_t)(sb.t_hi - sb.t_lo + 1);
+        const uint64_t gsegs = p.B / sb.seg;
+        seg_elems = std::max<uint64_t>(seg_elems, sw * gsegs);
+        const uint64_t nb_bits = (uint64_t)ilog2_u64(gsegs) + 1;           // NB + 1 sets
+        mid_elems = std::max<uint64_t>(mid_elems, sw * nb_bits * ((gsegs + RB_PER - 1) / RB_PER));
+        terms_elems = std::max<uint64_t>(terms_elems, sw * nb_bits);
+      }
       g.chunk_base = p.chunks_max;
       g.chunks_max = (n * wins + p.S - 1) / p.S + 1;
       // a heavy bucket spans > MERGE_QMAX chunks: at most chunks / MERGE_QMAX of them
@@ -536,10 +565,10 @@ struct Impl {
     const int ngroups = (int)p.groups.size();
     StreamCtx* ctx = nullptr;
     cudaStream_t ss = s, st2 = s;
-    if (ngroups > 1) {
+    if (ngroups > 1 || p.split_reduce) {
       if (gzkp_status st = stream_ctx(s, &ctx)) return st;
       if (ngroups > 16) return set_error(GZKP_ERROR_INVALID_VALUE, "too many window groups");
-      ss = ctx->side;
+      ss = ngroups > 1 ? ctx->side : s;
       st2 = ctx->side2;
     }
     const int threads = 128;
@@ -660,49 +689,56 @@ struct Impl {
       GZ_CHECK(cudaGetLastError());
       launches += 2 + gr.heavy_levels;
       ev_merged = profile_event(prof, ss);
-      // a6 (side stream): bucket reduction of the group's windows
-      const int gw = p.consolidated ? p.Wb : gr.t_hi - gr.t_lo + 1;
-      const int t_lo = p.consolidated ? 0 : gr.t_lo;
-      const uint32_t G = p.B / gr.seg;
-      const uint32_t total = (uint32_t)gw * G;
-      uint32_t* segT = U(p.o_seg);
-      uint32_t* segR = segT + p.seg_stride;
-      // small CTAs spread the ~W 2^(c-1) / s segment threads evenly over the
-      // SMs (32K threads on 148 SMs: 128-thread CTAs leave some SMs at 1 CTA)
-      static const int rcta = [] {
-        const char* e = getenv("GZKP_REDUCE_CTA");
-        const int v = e ? atoi(e) : 64;              // measured: 64 / 32 / 128 = 1.02 / 1.03 / 1.05 ms
-        return (v >= 32 && v <= 128 && v % 32 == 0) ? v : 64;
-      }();
-      k_reduce_seg<C><<<(total + rcta - 1) / rcta, rcta, 0, ss>>>(U(p.o_buckets), U(p.o_offsets), t_lo, gw,
-                                                                           p.B, gr.seg, segT, segR);
-      GZ_CHECK(cudaGetLastError());
-      const int NB = ilog2_u64(G);
-      const uint32_t nsl = (G + RB_PER - 1) / RB_PER;
-      const size_t rsmem = (size_t)RB_THREADS * 4 * N * 4;
-      const uint32_t nslR = (G / 2 + RB_PER - 1) / RB_PER;
-      k_reduce_bits<C><<<dim3(NB * nslR + nsl, gw), RB_THREADS, rsmem, ss>>>(segT, segR, G, NB, nsl, U(p.o_mid));
-      GZ_CHECK(cudaGetLastError());
-      k_reduce_bits_fin<C><<<dim3(NB + 1, gw), 32, 0, ss>>>(U(p.o_mid), G, NB, nsl, ilog2_u64(gr.seg), U(p.o_terms));
-      GZ_CHECK(cudaGetLastError());
-      k_reduce_bits_sum<C><<<gw, 32, 0, ss>>>(U(p.o_terms), NB, U(p.o_win) + (size_t)t_lo * 4 * N);
-      GZ_CHECK(cudaGetLastError());
-      launches += 4;
-      ev_reduced = profile_event(prof, ss);
-      // a7 (+ a8 on the last group): Horner over the group's windows, on its
-      // own stream so the next group's merge / reduction never queue behind
-      // this latency-bound chain (the chain itself runs group after group)
-      if (ctx) {
-        GZ_CHECK(cudaEventRecord(ctx->ev[16 + gi], ss));
-        GZ_CHECK(cudaStreamWaitEvent(st2, ctx->ev[16 + gi], 0));
+      // a6 (side stream): bucket reduction of the group's windows, by
+      // sub-group from the top; a7 (+ a8 on the last one): Horner over each
+      // sub-group's windows on side stream 2, so a sub-group's chain runs while
+      // the next sub-group is reduced and the next group merged (the chain
+      // itself runs sub-group after sub-group)
+      for (size_t k = 0; k < gr.subs.size(); ++k) {
+        const auto& sb = gr.subs[k];
+        const int gw = sb.t_hi - sb.t_lo + 1;
+        const int t_lo = sb.t_lo;
+        const uint32_t G = p.B / sb.seg;
+        const uint32_t total = (uint32_t)gw * G;
+        uint32_t* segT = U(p.o_seg);
+        uint32_t* segR = segT + p.seg_stride;
+        // small CTAs spread the ~W 2^(c-1) / s segment threads evenly over the
+        // SMs (32K threads on 148 SMs: 128-thread CTAs leave some SMs at 1 CTA)
+        static const int rcta = [] {
+          const char* e = getenv("GZKP_REDUCE_CTA");
+          const int v = e ? atoi(e) : 64;              // measured: 64 / 32 / 128 = 1.02 / 1.03 / 1.05 ms
+          return (v >= 32 && v <= 128 && v % 32 == 0) ? v : 64;
+        }();
+        k_reduce_seg<C><<<(total + rcta - 1) / rcta, rcta, 0, ss>>>(U(p.o_buckets), U(p.o_offsets), t_lo, gw,
+                                                                    p.B, sb.seg, segT, segR);
+        GZ_CHECK(cudaGetLastError());
+        const int NB = ilog2_u64(G);
+        const uint32_t nsl = (G + RB_PER - 1) / RB_PER;
+        const size_t rsmem = (size_t)RB_THREADS * 4 * N * 4;
+        const uint32_t nslR = (G / 2 + RB_PER - 1) / RB_PER;
+        k_reduce_bits<C><<<dim3(NB * nslR + nsl, gw), RB_THREADS, rsmem, ss>>>(segT, segR, G, NB, nsl, U(p.o_mid));
+        GZ_CHECK(cudaGetLastError());
+        k_reduce_bits_fin<C><<<dim3(NB + 1, gw), 32, 0, ss>>>(U(p.o_mid), G, NB, nsl, ilog2_u64(sb.seg),
+                                                              U(p.o_terms));
+        GZ_CHECK(cudaGetLastError());
+        k_reduce_bits_sum<C><<<gw, 32, 0, ss>>>(U(p.o_terms), NB, U(p.o_win) + (size_t)t_lo * 4 * N);
+        GZ_CHECK(cudaGetLastError());
+        launches += 4;
+        ev_reduced = profile_event(prof, ss);
+        if (ctx) {
+          const int evi = 16 + (int)(gi * 8 + k) % 40;
+          GZ_CHECK(cudaEventRecord(ctx->ev[evi], ss));
+          GZ_CHECK(cudaStreamWaitEvent(st2, ctx->ev[evi], 0));
+        }
+        const bool first = gi == 0 && k == 0;
+        const bool last = gi == ngroups - 1 && k + 1 == gr.subs.size();
+        k_tail<C><<<1, 32, 0, st2>>>(U(p.o_win), sb.t_hi, t_lo, p.c, first, last, U(p.o_state),
+                                    last ? (uint32_t*)call.out_partial : nullptr,
+                                    last ? (uint32_t*)call.out_affine : nullptr);
+        GZ_CHECK(cudaGetLastError());
+        ++launches;
+        ev_tailed = profile_event(prof, st2);
       }
-      const int last = gi == ngroups - 1;
-      k_tail<C><<<1, 32, 0, st2>>>(U(p.o_win), p.consolidated ? p.Wb - 1 : gr.t_hi, t_lo, p.c, gi == 0, last, U(p.o_state),
-                                  last ? (uint32_t*)call.out_partial : nullptr,
-                                  last ? (uint32_t*)call.out_affine : nullptr);
-      GZ_CHECK(cudaGetLastError());
-      ++launches;
-      ev_tailed = profile_event(prof, st2);
     }
     // phases 2-4 = the exposed post-processing of the last group
     profile_interval(prof, 2, ev_last_acc, ev_merged);

@@ -6,6 +6,8 @@ because the switches are read once per process:
 * GZKP_PIPELINE=2      two equal window groups
 * GZKP_ACCUM_THREADS=32  small accumulation CTAs
 * GZKP_WINDOW_BITS / GZKP_SEGMENT  planner overrides
+* GZKP_REDUCE_GROUPS=R  bucket reduction in R window sub-groups, the Horner
+                       tail of each on its own stream
 * GZKP_AFFINE_LEVELS=L  batch-affine tree levels before the XYZZ loop
                        (affine.cuh experiment; mnt4 and toy curves included)
 """
@@ -46,7 +48,9 @@ print("VARIANT_OK" if ok else "VARIANT_FAIL")
                                  {"GZKP_WINDOW_BITS": "11", "GZKP_SEGMENT": "5"},
                                  {"GZKP_DFP": "1", "GZKP_PIPELINE": "1", "GZKP_ACCUM_THREADS": "64"},
                                  {"GZKP_AFFINE_LEVELS": "3"}, {"GZKP_AFFINE_LEVELS": "12"},
-                                 {"GZKP_AFFINE_LEVELS": "2", "GZKP_WINDOW_BITS": "5"}],
+                                 {"GZKP_AFFINE_LEVELS": "2", "GZKP_WINDOW_BITS": "5"},
+                                 {"GZKP_REDUCE_GROUPS": "3"}, {"GZKP_REDUCE_GROUPS": "16"},
+                                 {"GZKP_REDUCE_GROUPS": "2", "GZKP_PIPELINE": "1"}],
                          ids=lambda e: ",".join(f"{k}={v}" for k, v in e.items()))
 def test_variant_parity(env):
     require_cuda()
