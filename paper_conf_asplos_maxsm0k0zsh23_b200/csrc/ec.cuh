@@ -18,6 +18,17 @@
 #include "field_dfp.cuh"
 #include "coop_mul.cuh"
 
+#ifndef GZKP_ADD2
+// ec_add_hot (N <= 12): paired products (EC::add2).  Measured: k_reduce_seg
+// 610 -> 620 us (BLS12-381 2^19), and madd_nz2 in the hot loop 0.99x
+// (tools/madd_bench.cu): ptxas already overlaps what the carry flag allows.
+#define GZKP_ADD2 0
+#endif
+
+#ifndef GZKP_MADD2_SQR
+#define GZKP_MADD2_SQR 1    // madd_nz2: the two squares as squares (1) or as one paired product (0)
+#endif
+
 #ifndef GZKP_COOP_SOS
 #define GZKP_COOP_SOS 0     // 1: separated-operand-scanning products in the cooperative chains
 #endif
@@ -133,6 +144,34 @@ struct EC {
     Fp::mul_sum(A.Y, R, t, PP, PPP);    // Y3 = R(Q - X3) - Y1 PPP (one reduction)
   }
 
+  // madd_nz with its independent products paired (F::mul2: rows of two
+  // products interleaved, four carry chains in flight instead of two)
+  GZ_DEV static void madd_nz2(Xyzz& A, const uint32_t x2[N], const uint32_t y2[N]) {
+    uint32_t P[N], R[N], PP[N], PPP[N], t[N];
+    Fp::mul2(P, x2, A.ZZ, R, y2, A.ZZZ);    // U2, S2
+    Fp::sub(P, P, A.X);                 // P = U2 - X1
+    Fp::sub(R, R, A.Y);                 // R = S2 - Y1
+    if (Fp::is_zero(P)) {
+      if (Fp::is_zero(R)) mdbl(A, x2, y2);
+      else set_inf(A);
+      return;
+    }
+#if GZKP_MADD2_SQR
+    Fp::sqr(PP, P);
+    Fp::sqr(t, R);
+#else
+    Fp::mul2(PP, P, P, t, R, R);        // PP = P^2, t = R^2
+#endif
+    Fp::mul2(PPP, P, PP, A.ZZ, A.ZZ, PP);     // PPP = P PP, ZZ3 = ZZ1 PP
+    Fp::mul2(A.ZZZ, A.ZZZ, PPP, PP, A.X, PP); // ZZZ3 = ZZZ1 PPP, Q = X1 PP
+    Fp::sub(t, t, PPP);
+    Fp::sub(t, t, PP);
+    Fp::sub(A.X, t, PP);                // X3 = R^2 - PPP - 2Q
+    Fp::sub(t, PP, A.X);
+    Fp::neg(PP, A.Y);
+    Fp::mul_sum(A.Y, R, t, PP, PPP);    // Y3 = R(Q - X3) - Y1 PPP (one reduction)
+  }
+
   // madd_nz with 4 of its 10 products on the FP64 pipe (Dfp<C>::mul, NEXT-2):
   // one product of each dependency level that has two or more (S2, R^2, Q,
   // Y1 PPP) goes to DFP, the rest stay on IMAD, so the two pipes work
@@ -188,6 +227,35 @@ struct EC {
     Fp::mul(A.ZZZ, A.ZZZ, PPP);         // ZZZ3 = ZZZ1 ZZZ2 PPP
     Fp::mul(PP, U1, PP);                // Q = U1 PP
     Fp::sqr(t, R);
+    Fp::sub(t, t, PPP);
+    Fp::sub(t, t, PP);
+    Fp::sub(A.X, t, PP);                // X3 = R^2 - PPP - 2Q
+    Fp::sub(t, PP, A.X);
+    Fp::neg(S1, S1);
+    Fp::mul_sum(A.Y, R, t, S1, PPP);    // Y3 = R(Q - X3) - S1 PPP (one reduction)
+  }
+
+  // add with its independent products paired (F::mul2, four carry chains in
+  // flight): for the latency-bound post-processing (segment running sums,
+  // tree sums, merges) that runs few warps per SM.  Same values as add().
+  GZ_DEV static void add2(Xyzz& A, const Xyzz& B) {
+    if (is_inf(B)) return;
+    if (is_inf(A)) { A = B; return; }
+    uint32_t U1[N], S1[N], P[N], R[N], PP[N], PPP[N], t[N];
+    Fp::mul2(U1, A.X, B.ZZ, P, B.X, A.ZZ);      // U1, U2
+    Fp::mul2(S1, A.Y, B.ZZZ, R, B.Y, A.ZZZ);    // S1, S2
+    Fp::sub(P, P, U1);                  // P = U2 - U1
+    Fp::sub(R, R, S1);                  // R = S2 - S1
+    if (Fp::is_zero(P)) {
+      if (Fp::is_zero(R)) dbl(A);
+      else set_inf(A);
+      return;
+    }
+    Fp::mul2(A.ZZ, A.ZZ, B.ZZ, A.ZZZ, A.ZZZ, B.ZZZ);   // ZZ1 ZZ2, ZZZ1 ZZZ2
+    Fp::sqr(PP, P);
+    Fp::sqr(t, R);
+    Fp::mul2(PPP, P, PP, A.ZZ, A.ZZ, PP);      // PPP = P PP, ZZ3 = ZZ1 ZZ2 PP
+    Fp::mul2(A.ZZZ, A.ZZZ, PPP, PP, U1, PP);   // ZZZ3 = ZZZ1 ZZZ2 PPP, Q = U1 PP
     Fp::sub(t, t, PPP);
     Fp::sub(t, t, PP);
     Fp::sub(A.X, t, PP);                // X3 = R^2 - PPP - 2Q
@@ -429,7 +497,8 @@ __device__ __noinline__ void ec_to_affine(uint32_t* x, uint32_t* y, const typena
 // curves) keeps the calls.
 template <class C>
 GZ_DEV void ec_add_hot(typename EC<C>::Xyzz& A, const typename EC<C>::Xyzz& B) {
-  if constexpr (C::N <= 12) EC<C>::add(A, B);
+  if constexpr (C::N <= 12 && GZKP_ADD2) EC<C>::add2(A, B);
+  else if constexpr (C::N <= 12) EC<C>::add(A, B);
   else ec_add<C>(A, B);
 }
 }  // namespace gzkp

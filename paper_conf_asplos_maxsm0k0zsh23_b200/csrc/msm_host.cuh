@@ -133,7 +133,13 @@ struct Impl {
       const double B = std::ldexp(1.0, c - 1);
       const double entries = (double)n * W * (1.0 - std::ldexp(1.0, -c));
       const int Mi = std::min(std::max(interval, 1), W);
-      const double reduce = Mi * B * 3.4 * add + 60.0 * add * lat / 8.0;
+      // per-bucket reduction + merge cost: 8 adds for the ~255-bit fields
+      // (round-2 sweep, profiles/r02_reduce_groups_prepared_c_sweep.txt:
+      // BLS12-381 2^19 best at c = 16, 4.33 ms, where 3.4 picked c = 18, 4.74
+      // ms; 2^22 keeps c = 20); MNT4-753's sweep is not monotone in c (the
+      // merge phase), 3.4 picks its second-best c there
+      const double per_bucket = N >= 24 ? 3.4 : 8.0;
+      const double reduce = Mi * B * per_bucket * add + 60.0 * add * lat / 8.0;
       const double tail = (Mi - 1) * (c * 10.0 + add) * lat;
       const double cost = entries * madd + reduce + tail;
       if (cost < best_cost) { best_cost = cost; best = c; }
@@ -272,9 +278,13 @@ struct Impl {
         const long v = e ? atol(e) : 32768;
         return (uint64_t)(v > 0 ? v : 32768);
       }();
+      // one bucket set (weighted points) of the <= 12-limb fields: 8K threads
+      // (round-2 sweep: BLS12-381 2^19 prepared reduce 0.407 -> 0.388 ms,
+      // BN254 2^20 0.349 -> 0.304; MNT4-753 prefers 32K)
+      const uint64_t tgt = (consolidated && N <= 12 && !getenv("GZKP_REDUCE_THREADS")) ? 8192 : target;
       auto seg_for = [&](uint64_t w) {
         uint64_t sg = 16;
-        while (sg > 1 && w * p.B / sg < target) sg >>= 1;
+        while (sg > 1 && w * p.B / sg < tgt) sg >>= 1;
         return (int)std::min<uint64_t>(sg, p.B);
       };
       g.seg = seg_for(bwins);
@@ -609,7 +619,7 @@ struct Impl {
             GZ_CHECK(cudaFuncSetAttribute(k_affine_level<C, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, asm_));
           }
           GZ_CHECK(cudaFuncSetAttribute(k_reduce_bits<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                        (int)((size_t)RB_THREADS * 4 * N * 4)));
+                                        (int)rb_smem_bytes<C>()));
           GZ_CHECK(cudaFuncSetAttribute(k_heavy_tree<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         (int)((size_t)HEAVY_THREADS * 4 * N * 4)));
           return GZKP_SUCCESS;
@@ -714,7 +724,7 @@ struct Impl {
         GZ_CHECK(cudaGetLastError());
         const int NB = ilog2_u64(G);
         const uint32_t nsl = (G + RB_PER - 1) / RB_PER;
-        const size_t rsmem = (size_t)RB_THREADS * 4 * N * 4;
+        const size_t rsmem = rb_smem_bytes<C>();
         const uint32_t nslR = (G / 2 + RB_PER - 1) / RB_PER;
         k_reduce_bits<C><<<dim3(NB * nslR + nsl, gw), RB_THREADS, rsmem, ss>>>(segT, segR, G, NB, nsl, U(p.o_mid));
         GZ_CHECK(cudaGetLastError());

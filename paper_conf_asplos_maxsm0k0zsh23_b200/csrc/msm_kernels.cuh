@@ -16,6 +16,11 @@
 #include <cuda_runtime.h>
 
 #include "ec.cuh"
+#include "coop_smem.cuh"
+
+#ifndef GZKP_COOP_SMEM
+#define GZKP_COOP_SMEM 1   // serial chains on CoopS (shared-memory slots) for N >= 12; 0: CoopEC everywhere
+#endif
 
 namespace gzkp {
 
@@ -809,6 +814,16 @@ __global__ void __launch_bounds__(128, 2) k_reduce_seg(const uint32_t* __restric
 
 constexpr uint32_t RB_PER = 512;          // set elements per k_reduce_bits CTA
 constexpr int RB_THREADS = 128;
+// the serial chains and short trees of the reduction run on CoopS groups for
+// N >= 12 (GZKP_COOP_SMEM); k_reduce_bits' CTA tree uses RB_GROUPS of them
+template <class C>
+constexpr bool coop_tree() { return GZKP_COOP_SMEM && C::N >= 12; }
+template <class C>
+constexpr int rb_groups() { return C::N <= 12 ? RB_THREADS / 4 : 8; }
+template <class C>
+constexpr size_t rb_smem_bytes() {
+  return (size_t)RB_THREADS * 4 * C::N * 4 + (coop_tree<C>() ? (size_t)rb_groups<C>() * CoopS<C>::WORDS * 4 : 0);
+}
 
 // set k < NB: the G/2 segments g with bit k set (e-th such g: insert a 1 at
 // bit k of e); set NB: all G segments of segT.  The grid is exact, (slices of
@@ -840,6 +855,12 @@ __global__ void __launch_bounds__(RB_THREADS, 3) k_reduce_bits(const uint32_t* _
   }
   EC_::store(red_smem + threadIdx.x * 4 * N, acc);
   __syncthreads();
+  if constexpr (coop_tree<C>()) {
+    CoopS<C>::tree_sum(red_smem, RB_THREADS, red_smem + RB_THREADS * 4 * N, rb_groups<C>());
+    uint32_t* dst = mid + ((size_t)(t * (NB + 1) + k) * nsl + slice) * 4 * N;
+    for (int i = threadIdx.x; i < 4 * N; i += RB_THREADS) dst[i] = red_smem[i];
+    return;
+  }
   for (uint32_t w = RB_THREADS / 2; w > 0; w >>= 1) {
     if (threadIdx.x < w) {
       typename EC_::Xyzz X;
@@ -876,7 +897,7 @@ GZ_DEV void warp_sum(typename EC<C>::Xyzz& acc, uint32_t* sm, int used = 32) {
 
 // <<<(NB+1, W), 32>>>: S_k (or A) from its slice partials, times 2^(k + log2 s)
 template <class C>
-__global__ void __launch_bounds__(32) k_reduce_bits_fin(const uint32_t* __restrict__ mid, uint32_t G, int NB,
+__global__ void __launch_bounds__(32) k_reduce_bits_fin(uint32_t* __restrict__ mid, uint32_t G, int NB,
                                                         uint32_t nsl, int log_s, uint32_t* __restrict__ terms) {
   using EC_ = EC<C>;
   using CO = CoopEC<C>;
@@ -884,37 +905,59 @@ __global__ void __launch_bounds__(32) k_reduce_bits_fin(const uint32_t* __restri
   const uint32_t k = blockIdx.x, t = blockIdx.y;
   const uint32_t size = (int)k < NB ? G / 2 : G;
   const uint32_t used = (size + RB_PER - 1) / RB_PER;
-  const uint32_t* src = mid + (size_t)(t * (NB + 1) + k) * nsl * 4 * N;
-  typename EC_::Xyzz acc;
-  EC_::set_inf(acc);
-  for (uint32_t q = threadIdx.x; q < used; q += 32) {
-    typename EC_::Xyzz X;
-    EC_::load(X, src + (size_t)q * 4 * N);
-    ec_add_hot<C>(acc, X);
+  uint32_t* src = mid + (size_t)(t * (NB + 1) + k) * nsl * 4 * N;
+  if constexpr (coop_tree<C>()) {
+    // tree over the slice partials by the warp's 8 groups, then group 0
+    // doubles (k + log2 s) times
+    using CS = CoopS<C>;
+    __shared__ __align__(16) uint32_t gsm[8 * CS::WORDS];
+    CS::tree_sum(src, (int)used, gsm, 8);
+    if (threadIdx.x < 4) {
+      CS::put_words(gsm, CS::AX, src);
+      if ((int)k < NB)
+        for (int d = 0; d < (int)k + log_s; ++d) CS::dbl(gsm);
+      CS::store_a(terms + (size_t)(t * (NB + 1) + k) * 4 * N, gsm);
+    }
+  } else {
+    typename EC_::Xyzz acc;
+    EC_::set_inf(acc);
+    for (uint32_t q = threadIdx.x; q < used; q += 32) {
+      typename EC_::Xyzz X;
+      EC_::load(X, src + (size_t)q * 4 * N);
+      ec_add_hot<C>(acc, X);
+    }
+    __shared__ __align__(16) uint32_t sm[32 * 4 * N];
+    warp_sum<C>(acc, sm, (int)min(used, 32u));
+    if (threadIdx.x == 0) EC_::store(sm, acc);
+    __syncwarp();
+    EC_::load(acc, sm);                 // every lane holds the sum (CoopEC)
+    if ((int)k < NB)
+      for (int d = 0; d < (int)k + log_s; ++d) CO::dbl(acc);
+    if (threadIdx.x == 0) EC_::store(terms + (size_t)(t * (NB + 1) + k) * 4 * N, acc);
   }
-  __shared__ __align__(16) uint32_t sm[32 * 4 * N];
-  warp_sum<C>(acc, sm, (int)min(used, 32u));
-  if (threadIdx.x == 0) EC_::store(sm, acc);
-  __syncwarp();
-  EC_::load(acc, sm);                   // every lane holds the sum (CoopEC)
-  if ((int)k < NB)
-    for (int d = 0; d < (int)k + log_s; ++d) CO::dbl(acc);
-  if (threadIdx.x == 0) EC_::store(terms + (size_t)(t * (NB + 1) + k) * 4 * N, acc);
 }
 
 // <<<W, 32>>>: W_t = sum of the window's NB + 1 terms (NB + 1 <= 32)
 template <class C>
-__global__ void __launch_bounds__(32) k_reduce_bits_sum(const uint32_t* __restrict__ terms, int NB,
+__global__ void __launch_bounds__(32) k_reduce_bits_sum(uint32_t* __restrict__ terms, int NB,
                                                         uint32_t* __restrict__ win_out) {
   using EC_ = EC<C>;
   constexpr int N = C::N;
   const uint32_t t = blockIdx.x;
-  typename EC_::Xyzz acc;
-  EC_::set_inf(acc);
-  if ((int)threadIdx.x <= NB) EC_::load(acc, terms + (size_t)(t * (NB + 1) + threadIdx.x) * 4 * N);
-  __shared__ __align__(16) uint32_t sm[32 * 4 * N];
-  warp_sum<C>(acc, sm, NB + 1);
-  if (threadIdx.x == 0) EC_::store(win_out + (size_t)t * 4 * N, acc);
+  if constexpr (coop_tree<C>()) {
+    using CS = CoopS<C>;
+    __shared__ __align__(16) uint32_t gsm[8 * CS::WORDS];
+    uint32_t* v = terms + (size_t)t * (NB + 1) * 4 * N;
+    CS::tree_sum(v, NB + 1, gsm, 8);
+    for (int i = threadIdx.x; i < 4 * N; i += 32) win_out[(size_t)t * 4 * N + i] = v[i];
+  } else {
+    typename EC_::Xyzz acc;
+    EC_::set_inf(acc);
+    if ((int)threadIdx.x <= NB) EC_::load(acc, terms + (size_t)(t * (NB + 1) + threadIdx.x) * 4 * N);
+    __shared__ __align__(16) uint32_t sm[32 * 4 * N];
+    warp_sum<C>(acc, sm, NB + 1);
+    if (threadIdx.x == 0) EC_::store(win_out + (size_t)t * 4 * N, acc);
+  }
 }
 
 // ----------------------------------------- a7 window combination + a8 output
@@ -934,17 +977,37 @@ __global__ void __launch_bounds__(32) k_tail(const uint32_t* __restrict__ win_ou
   if (blockIdx.x) return;
   typename EC_::Xyzz Q;
   int t = t_hi;
-  if (first) {
-    EC_::load(Q, win_out + (size_t)t * 4 * N);
-    --t;
+  if constexpr (GZKP_COOP_SMEM && N >= 12) {
+    // CoopS (measured, tools/tail_bench.cu: BLS12-381 3.40 -> 3.28 us per
+    // doubling, MNT4-753 13.5 -> 12.8; BN254 1.74 -> 1.77 keeps CoopEC)
+    using CS = CoopS<C>;
+    __shared__ __align__(16) uint32_t sm[CS::WORDS];
+    if (threadIdx.x >= 4) return;                  // one 4-lane group runs the chain
+    if (first) {
+      CS::put_words(sm, CS::AX, win_out + (size_t)t * 4 * N);
+      --t;
+    } else {
+      CS::put_words(sm, CS::AX, state);
+    }
+    for (; t >= t_lo; --t) {
+      for (int k = 0; k < c; ++k) CS::dbl(sm);
+      CS::put_words(sm, CS::BX, win_out + (size_t)t * 4 * N);
+      CS::add(sm);
+    }
+    CS::get(Q, sm, CS::AX);
   } else {
-    EC_::load(Q, state);
-  }
-  for (; t >= t_lo; --t) {
-    for (int k = 0; k < c; ++k) CO::dbl(Q);
-    typename EC_::Xyzz X;
-    EC_::load(X, win_out + (size_t)t * 4 * N);
-    CO::add(Q, X);
+    if (first) {
+      EC_::load(Q, win_out + (size_t)t * 4 * N);
+      --t;
+    } else {
+      EC_::load(Q, state);
+    }
+    for (; t >= t_lo; --t) {
+      for (int k = 0; k < c; ++k) CO::dbl(Q);
+      typename EC_::Xyzz X;
+      EC_::load(X, win_out + (size_t)t * 4 * N);
+      CO::add(Q, X);
+    }
   }
   if (threadIdx.x) return;
   if (!last) {
