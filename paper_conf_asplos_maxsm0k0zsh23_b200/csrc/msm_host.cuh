@@ -424,7 +424,8 @@ struct Impl {
   // histogram, exclusive scan -> offsets[0..M] (offsets[M] = E), and the
   // scatter of (point index | sign) into bucket order -> vals[0..E).
   static gzkp_status sort_stage(const MsmCall& call, const Plan& p, char* ws, int* launches,
-                                const uint32_t* scalars = nullptr, const uint32_t* rng = nullptr) {
+                                const uint32_t* scalars = nullptr, const uint32_t* rng = nullptr,
+                                const uint32_t* remap = nullptr) {
     cudaStream_t s = call.stream;
     const size_t n = call.n;
     auto U = [&](size_t off) { return (uint32_t*)(ws + off); };
@@ -452,10 +453,10 @@ struct Impl {
     const uint32_t bpw_s = (uint32_t)((n + SCATTER_TILE - 1) / SCATTER_TILE);
     k_scatter<<<(unsigned)((uint64_t)bpw_s * p.W), SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw_s, p.B, (uint32_t)p.Mi,
                                                                          p.val_stride, U(p.o_hot), U(p.o_cursor), U(p.o_vals),
-                                                                         rng);
+                                                                         rng, remap);
     if (rng)
       k_scatter<<<bpw_s, SCATTER_THREADS, 0, s>>>(U(p.o_codes), n, bpw_s, p.B, (uint32_t)p.Mi, p.val_stride, U(p.o_hot),
-                                                  U(p.o_cursor), U(p.o_vals), rng + 2);
+                                                  U(p.o_cursor), U(p.o_vals), rng + 2, remap);
     GZ_CHECK(cudaGetLastError());
     *launches += 5;
     return GZKP_SUCCESS;
@@ -545,10 +546,32 @@ struct Impl {
     int launches = 0;
     const int sms = device_sm_count();
 
-    // a1: points -> Montgomery (skipped for prepared handles)
+    // NEXT-2's mixed hot loop (GZKP_DFP=1), the 3-CTA build and the
+    // batch-affine levels read Montgomery points, and so does the default;
+    // GZKP_CANON=1 reads the caller's canonical points directly
+    static const bool mixed = [] {
+      const char* e = getenv("GZKP_DFP");
+      return AccumCfg<C>::DFP && (e ? atoi(e) != 0 : AccumCfg<C>::DFP_DEFAULT);
+    }();
+    // GZKP_ACCUM_MINB=3: the BLS12-381 hot loop compiled for 3 CTAs / SM
+    static const bool minb3 = [] {
+      const char* e = getenv("GZKP_ACCUM_MINB");
+      return AccumCfg<C>::DFP && e && atoi(e) == 3;
+    }();
+    // GZKP_CANON=1: the canonical-input hot loop (Canon, msm_kernels.cuh) --
+    // no conversion pass, but each run start / flush does 1 / 2 products on
+    // a divergent lane; measured slower (BLS12-381 2^22 accumulation 24.2 ->
+    // 42.2 ms, ncu: no_instruction stalls 0.17M -> 1.53M samples), so off
+    static const bool canon_env = [] {
+      const char* e = getenv("GZKP_CANON");
+      return e ? atoi(e) != 0 : false;
+    }();
+    const bool canon = Canon<C>::ON && canon_env && !call.prepared && !mixed && !minb3 && p.aff_levels == 0;
+    // a1: points -> Montgomery (skipped for prepared handles and the canonical hot loop)
     const uint32_t* pts = (const uint32_t*)call.points;
     const uint32_t* sc_sorted = nullptr;
     const uint32_t* rng = nullptr;
+    const uint32_t* remap = nullptr;
     if (!call.prepared) {
       // drop the zero scalars (small ones to the back), then convert the
       // remaining points in the compacted order
@@ -556,16 +579,21 @@ struct Impl {
       k_compact<C><<<(unsigned)((n + 255) / 256), 256, 0, s>>>((const uint32_t*)call.scalars, n, p.c, U(p.o_scc),
                                                               U(p.o_idx), U(p.o_ncnt));
       k_compact_ranges<<<1, 1, 0, s>>>(U(p.o_ncnt), (uint32_t)n, U(p.o_ncnt) + 2);
-      const int cgrid = (int)std::min<size_t>((n + 255) / 256, (size_t)sms * 16);
-      k_to_mont_c<C><<<cgrid, 256, 0, s>>>((const uint32_t*)call.points, U(p.o_idx), U(p.o_ncnt) + 2, U(p.o_pts));
+      if (canon) {
+        remap = U(p.o_idx);                  // entries name the original point
+      } else {
+        const int cgrid = (int)std::min<size_t>((n + 255) / 256, (size_t)sms * 16);
+        k_to_mont_c<C><<<cgrid, 256, 0, s>>>((const uint32_t*)call.points, U(p.o_idx), U(p.o_ncnt) + 2, U(p.o_pts));
+        pts = U(p.o_pts);
+        ++launches;
+      }
       GZ_CHECK(cudaGetLastError());
-      pts = U(p.o_pts);
       sc_sorted = U(p.o_scc);
       rng = U(p.o_ncnt) + 2;
-      launches += 5;
+      launches += 4;
     }
     // a2 + a3: signed digits, bucket histogram, offsets, sort by bucket
-    if (gzkp_status st = sort_stage(call, p, ws, &launches, sc_sorted, rng)) return st;
+    if (gzkp_status st = sort_stage(call, p, ws, &launches, sc_sorted, rng, remap)) return st;
     cudaEvent_t ev_sorted = profile_event(prof, s);
     profile_interval(prof, 0, ev_begin, ev_sorted);
 
@@ -590,20 +618,16 @@ struct Impl {
       return (v >= 32 && v <= 128 && v % 32 == 0) ? v : AccumCfg<C>::THREADS;
     }();
     const size_t acc_smem = (size_t)acc_threads * Stage<C>::SLOT_WORDS * 4;
-    // NEXT-2: the hot loop with 4 of 10 products on the FP64 pipe (BLS12-381)
-    static const bool mixed = [] {
-      const char* e = getenv("GZKP_DFP");
-      return AccumCfg<C>::DFP && (e ? atoi(e) != 0 : AccumCfg<C>::DFP_DEFAULT);
-    }();
-    // GZKP_ACCUM_MINB=3: the BLS12-381 hot loop compiled for 3 CTAs / SM
-    static const bool minb3 = [] {
-      const char* e = getenv("GZKP_ACCUM_MINB");
-      return AccumCfg<C>::DFP && e && atoi(e) == 3;
-    }();
+    // NEXT-2: the hot loop with 4 of 10 products on the FP64 pipe (BLS12-381): `mixed` above
+
     static int attr_tag;   // kernel attributes are per device
     if (gzkp_status st = once_per_device(&attr_tag, [] {
           GZ_CHECK(cudaFuncSetAttribute(k_accum<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
+          if constexpr (Canon<C>::ON)
+            GZ_CHECK(cudaFuncSetAttribute(k_accum<C, false, AccumCfg<C>::MIN_CTAS, false, true>,
+                                          cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
           if constexpr (AccumCfg<C>::DFP)
             GZ_CHECK(cudaFuncSetAttribute(k_accum<C, false, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                           (int)((size_t)128 * Stage<C>::SLOT_WORDS * 4)));
@@ -659,6 +683,16 @@ struct Impl {
         else if (minb3)
           k_accum<C, false, 3><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
                                                                        U(p.o_buckets), U(p.o_spay), mlist, mcnt);
+        else if (canon)
+          k_accum<C, false, AccumCfg<C>::MIN_CTAS, false, true><<<acc_grid, acc_threads, acc_smem, s>>>(
+              U(p.o_vals), U(p.o_offsets), grp, pts, p.S, U(p.o_buckets), U(p.o_spay), mlist, mcnt);
+        else
+          k_accum<C><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
+                                                             U(p.o_buckets), U(p.o_spay), mlist, mcnt);
+      } else if constexpr (Canon<C>::ON) {
+        if (canon)
+          k_accum<C, false, AccumCfg<C>::MIN_CTAS, false, true><<<acc_grid, acc_threads, acc_smem, s>>>(
+              U(p.o_vals), U(p.o_offsets), grp, pts, p.S, U(p.o_buckets), U(p.o_spay), mlist, mcnt);
         else
           k_accum<C><<<acc_grid, acc_threads, acc_smem, s>>>(U(p.o_vals), U(p.o_offsets), grp, pts, p.S,
                                                              U(p.o_buckets), U(p.o_spay), mlist, mcnt);

@@ -332,7 +332,10 @@ static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32
                                                              uint32_t bpw, uint32_t B, uint32_t Mi, uint32_t val_stride,
                                                              const uint32_t* __restrict__ hotbits,
                                                              uint32_t* __restrict__ cursor, uint32_t* __restrict__ vals,
-                                                             const uint32_t* __restrict__ rng) {
+                                                             const uint32_t* __restrict__ rng,
+                                                             const uint32_t* __restrict__ remap) {
+  // remap (may be null): entry value = remap[i] (the compacted point's
+  // original index, for the canonical-input hot loop) instead of i
   // codes exist for i in [lo, hi) (rng, device; null = [0, n)), row stride n
   __shared__ uint32_t s_key[HOT_SLOTS], s_cnt[HOT_SLOTS], s_base[HOT_SLOTS];
   const int tid = threadIdx.x;
@@ -394,7 +397,8 @@ static __global__ void __launch_bounds__(SCATTER_THREADS) k_scatter(const uint32
         if (lane == leader[q] && h[q] >= 0) p += s_base[h[q]];
         p = __shfl_sync(peers[q], p, leader[q]) + __popc(peers[q] & ((1u << lane) - 1u));
       }
-      vals[p] = (vbase + (uint32_t)(i0 + q)) | (code[q] & VAL_NEG);
+      const uint32_t pi = remap ? __ldg(remap + i0 + q) : (uint32_t)(i0 + q);
+      vals[p] = (vbase + pi) | (code[q] & VAL_NEG);
     }
   }
 }
@@ -533,6 +537,95 @@ GZ_DEV uint32_t find_bucket(const uint32_t* __restrict__ off, uint32_t lo, uint3
   return lo;
 }
 
+// ---- canonical input points in the hot loop (no Montgomery conversion pass;
+// GZKP_CANON=1 experiment, off: the per-run products below run on divergent
+// lanes and cost more than the conversion pass saves)
+// The affine input (x2, y2) enters madd only through U2 = x2 ZZ1 and
+// S2 = y2 ZZZ1.  If the accumulator keeps ZZ and ZZZ "primed" -- the
+// Montgomery representation of ZZ R and ZZZ R instead of ZZ and ZZZ -- then
+// the Montgomery product of the raw canonical x2 with the primed ZZ1 is
+// x2 ZZ1 R R / R = (x2 ZZ1) R, the ordinary Montgomery form of U2, and the
+// products ZZ3 = ZZ1 PP, ZZZ3 = ZZZ1 PPP stay primed; X and Y are ordinary.
+// A run starts from the representative with Z = lambda = 2^(-16N) (lambda^2 =
+// 1/R): X = x (raw), Y = mont(y, K) = y lambda, ZZ' = R mod p (ONE),
+// ZZZ' = lambda R mod p = K, K = 2^(16N) mod p -- one product per run instead
+// of two conversions per point.  flush() returns ZZ, ZZZ to ordinary form
+// (one REDC each), so buckets and partials leave in the usual XYZZ form.
+template <class C>
+struct Canon {
+  static constexpr int N = C::N;
+  static constexpr bool ON = std::is_same<Field<C>, F<C>>::value;   // G1 (F_p) curves
+  GZ_DEV static void k_const(uint32_t k[N]) {
+#pragma unroll
+    for (int i = 0; i < N; ++i) k[i] = 0;
+    if constexpr (16 * N < C::P_BITS) {
+      k[(16 * N) / 32] = 1u << ((16 * N) % 32);
+    } else {                            // the toy curves: p < 2^32, N = 2
+      static_assert(N == 2, "canonical start constant");
+      const uint64_t p = (uint64_t)C::P(0) | ((uint64_t)C::P(1) << 32);
+      const uint64_t w = (1ull << 32) % p;                     // 2^(16N), 16N = 32
+      k[0] = (uint32_t)w;
+      k[1] = (uint32_t)(w >> 32);
+    }
+  }
+  // run start: the affine canonical point (x, y) as a primed XYZZ point
+  GZ_DEV static void start(typename EC<C>::Xyzz& A, const uint32_t x[N], const uint32_t y[N]) {
+    using Fp = F<C>;
+    uint32_t k[N];
+    k_const(k);
+    Fp::copy(A.X, x);
+    Fp::mul(A.Y, y, k);
+#pragma unroll
+    for (int i = 0; i < N; ++i) { A.ZZ[i] = C::ONE(i); A.ZZZ[i] = k[i]; }
+  }
+  // primed <-> ordinary ZZ, ZZZ
+  GZ_DEV static void unprime(typename EC<C>::Xyzz& A) {
+    using Fp = F<C>;
+    Fp::from_mont(A.ZZ, A.ZZ);
+    Fp::from_mont(A.ZZZ, A.ZZZ);
+  }
+  GZ_DEV static void prime(typename EC<C>::Xyzz& A) {
+    using Fp = F<C>;
+    Fp::to_mont(A.ZZ, A.ZZ);
+    Fp::to_mont(A.ZZZ, A.ZZZ);
+  }
+  // madd_nz on a primed accumulator with a canonical affine point; the
+  // exceptional same-point case doubles the (equal) accumulator instead
+  GZ_DEV static void madd(typename EC<C>::Xyzz& A, const uint32_t x2[N], const uint32_t y2[N]) {
+    using Fp = F<C>;
+    using E = EC<C>;
+    uint32_t P[N], R[N], PP[N], PPP[N], t[N];
+    Fp::mul(P, x2, A.ZZ);               // U2 (ordinary form, see above)
+    Fp::sub(P, P, A.X);
+    Fp::mul(R, y2, A.ZZZ);              // S2
+    Fp::sub(R, R, A.Y);
+    if (Fp::is_zero(P)) {
+      if (Fp::is_zero(R)) {             // same point: 2 A = 2 (x2, y2), inline like madd_nz's mdbl
+        uint32_t xm[N], ym[N];
+        Fp::to_mont(xm, x2);
+        Fp::to_mont(ym, y2);
+        E::mdbl(A, xm, ym);
+        prime(A);
+      } else {
+        E::set_inf(A);
+      }
+      return;
+    }
+    Fp::sqr(PP, P);
+    Fp::mul(PPP, P, PP);
+    Fp::mul(A.ZZ, A.ZZ, PP);            // ZZ3' = ZZ1' PP   (stays primed)
+    Fp::mul(A.ZZZ, A.ZZZ, PPP);         // ZZZ3' = ZZZ1' PPP
+    Fp::mul(PP, A.X, PP);               // Q = X1 PP
+    Fp::sqr(t, R);
+    Fp::sub(t, t, PPP);
+    Fp::sub(t, t, PP);
+    Fp::sub(A.X, t, PP);                // X3 = R^2 - PPP - 2Q
+    Fp::sub(t, PP, A.X);
+    Fp::neg(PP, A.Y);
+    Fp::mul_sum(A.Y, R, t, PP, PPP);    // Y3 = R(Q - X3) - Y1 PPP
+  }
+};
+
 // CTAs per SM the hot loop is compiled for (registers: 128 / 168 / 255 per
 // thread).  BN254 fits 3 CTAs in 168 registers; for BLS12-381 forcing 3 CTAs
 // (166 regs) measured slower than the unconstrained 2 CTAs (85.6 % IMAD pipe).
@@ -554,7 +647,9 @@ struct AccumCfg {
 // DIRECT: the entries are the points themselves (entry j = point j of `pts`,
 // no index array, no sign): the residual level array of the batch-affine
 // levels (affine.cuh).
-template <class C, bool MIXED = false, int MINB = AccumCfg<C>::MIN_CTAS, bool DIRECT = false>
+// CANON: `pts` holds the canonical input points (indexed by the entries'
+// original point index) instead of their Montgomery forms (Canon above).
+template <class C, bool MIXED = false, int MINB = AccumCfg<C>::MIN_CTAS, bool DIRECT = false, bool CANON = false>
 __global__ void __launch_bounds__(128, MINB)
     k_accum(const uint32_t* __restrict__ vals, const uint32_t* __restrict__ off, Group grp,
             const uint32_t* __restrict__ pts, int S, uint32_t* __restrict__ buckets, uint32_t* __restrict__ spay,
@@ -583,6 +678,7 @@ __global__ void __launch_bounds__(128, MINB)
     const bool open_l = first_run && __ldg(off + cur) < beg;
     const bool open_r = last_run && nxt > end;
     if (acc_inf) EC_::set_inf(acc);
+    else if constexpr (CANON) Canon<C>::unprime(acc);
     if (!open_l && !open_r) EC_::store(buckets + (size_t)cur * 4 * N, acc);
     else EC_::store(spay + (size_t)(open_l ? sidx : sidx + 1) * 4 * N, acc);
   };
@@ -611,10 +707,12 @@ __global__ void __launch_bounds__(128, MINB)
     if (Fp::is_zero(x) && Fp::is_zero(y)) continue;     // identity input point
     if (v & VAL_NEG) Fp::neg(y, y);
     if (acc_inf) {
-      EC_::from_affine(acc, x, y);
+      if constexpr (CANON) Canon<C>::start(acc, x, y);
+      else EC_::from_affine(acc, x, y);
       acc_inf = false;
     } else {
-      if constexpr (MIXED) EC_::madd_nz_mixed(acc, x, y);   // IMAD + FP64 pipes (NEXT-2)
+      if constexpr (CANON) Canon<C>::madd(acc, x, y);
+      else if constexpr (MIXED) EC_::madd_nz_mixed(acc, x, y);   // IMAD + FP64 pipes (NEXT-2)
       else EC_::madd_nz(acc, x, y);
       acc_inf = EC_::is_inf(acc);
     }
