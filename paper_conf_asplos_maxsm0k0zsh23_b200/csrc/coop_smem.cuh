@@ -35,7 +35,9 @@ struct CoopS {
   // slots (N words each); the accumulator is A, an addend B
   enum : int {
     AX, AY, AZZ, AZZZ, BX, BY, BZZ, BZZZ,
-    U, V, XX, W, S, MM, M, T, R, PP, PPP, Q, T1, T2, S1, Z4, NSLOT
+    U, V, XX, W, S, MM, M, T, R, PP, PPP, Q, T1, T2, S1, Z4,
+    CX, CY, CZZ, CZZZ,            // a third point (k_reduce_seg's running sum T)
+    NSLOT
   };
   static constexpr int WORDS = NSLOT * N;      // per warp
 
@@ -87,18 +89,19 @@ struct CoopS {
     if (lane() == 0) E::st(at(sm, d), v);
   }
 
-  // A = 2A (dbl-2008-s-1, general a)
-  GZ_DEV static void dbl(uint32_t* sm) {
+  // A = 2A (slots a .. a+3) (dbl-2008-s-1, general a)
+  GZ_DEV static void dbl(uint32_t* sm, int a = AX) {
+    const int aX = a, aY = a + 1, aZZ = a + 2, aZZZ = a + 3;
     {
       uint32_t y[N], u[N];
-      E::ld(y, at(sm, AY));
+      E::ld(y, at(sm, aY));
       Fp::dbl(u, y);
       store0(sm, U, u);
       sync();
     }
     // V = U^2, XX = X^2 (, Z4 = ZZ^2)
-    if constexpr (C::A_ZERO) level<2, true>(sm, V, U, U, XX, AX, AX);
-    else level<3, true>(sm, V, U, U, XX, AX, AX, Z4, AZZ, AZZ);
+    if constexpr (C::A_ZERO) level<2, true>(sm, V, U, U, XX, aX, aX);
+    else level<3, true>(sm, V, U, U, XX, aX, aX, Z4, aZZ, aZZ);
     {
       uint32_t xx[N], m[N];
       E::ld(xx, at(sm, XX));
@@ -121,7 +124,7 @@ struct CoopS {
       sync();
     }
     // W = U V, S = X V, MM = M^2, ZZ3 = V ZZ
-    level<4>(sm, W, U, V, S, AX, V, MM, M, M, AZZ, V, AZZ);
+    level<4>(sm, W, U, V, S, aX, V, MM, M, M, aZZ, V, aZZ);
     {
       uint32_t mm[N], s[N], x3[N], t[N];
       E::ld(mm, at(sm, MM));
@@ -129,18 +132,18 @@ struct CoopS {
       Fp::sub(t, mm, s);
       Fp::sub(x3, t, s);                // X3 = M^2 - 2S
       Fp::sub(t, s, x3);
-      store0(sm, AX, x3);
+      store0(sm, aX, x3);
       store0(sm, T, t);
       sync();
     }
     // T = M (S - X3), S = W Y, ZZZ3 = W ZZZ
-    level<3>(sm, T, M, T, S, W, AY, AZZZ, W, AZZZ);
+    level<3>(sm, T, M, T, S, W, aY, aZZZ, W, aZZZ);
     {
       uint32_t a[N], b[N], y3[N];
       E::ld(a, at(sm, T));
       E::ld(b, at(sm, S));
       Fp::sub(y3, a, b);                // Y3 = M(S - X3) - W Y
-      store0(sm, AY, y3);
+      store0(sm, aY, y3);
       sync();
     }
   }
@@ -154,24 +157,26 @@ struct CoopS {
     for (int i = lane(); i < N; i += 4) sm[d * N + i] = sm[s * N + i];
     sync();
   }
-  GZ_DEV static void set_inf_a(uint32_t* sm) {
+  GZ_DEV static void set_inf_a(uint32_t* sm, int a = AX) {
     if (lane() == 0) {
       Xyzz O;
       E::set_inf(O);
-      E::st(at(sm, AX), O.X); E::st(at(sm, AY), O.Y); E::st(at(sm, AZZ), O.ZZ); E::st(at(sm, AZZZ), O.ZZZ);
+      E::st(at(sm, a), O.X); E::st(at(sm, a + 1), O.Y); E::st(at(sm, a + 2), O.ZZ); E::st(at(sm, a + 3), O.ZZZ);
     }
     sync();
   }
 
-  // A += B (add-2008-s), all cases; B in slots BX..BZZZ
-  GZ_DEV static void add(uint32_t* sm) {
-    if (is_zero_slot(sm, BZZ)) return;
-    if (is_zero_slot(sm, AZZ)) {
-      for (int s = 0; s < 4; ++s) copy_slot(sm, AX + s, BX + s);
+  // A += B (add-2008-s), all cases; A in slots a .. a+3, B in b .. b+3
+  GZ_DEV static void add(uint32_t* sm, int a = AX, int b = BX) {
+    const int aX = a, aY = a + 1, aZZ = a + 2, aZZZ = a + 3;
+    const int bX = b, bY = b + 1, bZZ = b + 2, bZZZ = b + 3;
+    if (is_zero_slot(sm, bZZ)) return;
+    if (is_zero_slot(sm, aZZ)) {
+      for (int s = 0; s < 4; ++s) copy_slot(sm, aX + s, bX + s);
       return;
     }
     // U1 = X1 ZZ2, U2 = X2 ZZ1, S1 = Y1 ZZZ2, S2 = Y2 ZZZ1
-    level<4>(sm, U, AX, BZZ, PP, BX, AZZ, S1, AY, BZZZ, R, BY, AZZZ);
+    level<4>(sm, U, aX, bZZ, PP, bX, aZZ, S1, aY, bZZZ, R, bY, aZZZ);
     bool pz, rz;
     {
       uint32_t u1[N], u2[N], s1[N], s2[N], p[N], r[N];
@@ -186,14 +191,14 @@ struct CoopS {
       sync();
     }
     if (pz) {
-      if (rz) dbl(sm);
-      else set_inf_a(sm);
+      if (rz) dbl(sm, aX);
+      else set_inf_a(sm, aX);
       return;
     }
     // PP = P^2, RR = R^2 (-> MM), T1 = ZZ1 ZZ2, T2 = ZZZ1 ZZZ2
-    level<4>(sm, PP, V, V, MM, R, R, T1, AZZ, BZZ, T2, AZZZ, BZZZ);
+    level<4>(sm, PP, V, V, MM, R, R, T1, aZZ, bZZ, T2, aZZZ, bZZZ);
     // PPP = P PP, Q = U1 PP, ZZ3 = T1 PP
-    level<3>(sm, PPP, V, PP, Q, U, PP, AZZ, T1, PP);
+    level<3>(sm, PPP, V, PP, Q, U, PP, aZZ, T1, PP);
     {
       uint32_t rr[N], ppp[N], q[N], t[N], x3[N];
       E::ld(rr, at(sm, MM)); E::ld(ppp, at(sm, PPP)); E::ld(q, at(sm, Q));
@@ -201,22 +206,27 @@ struct CoopS {
       Fp::sub(t, t, q);
       Fp::sub(x3, t, q);                // X3 = R^2 - PPP - 2Q
       Fp::sub(t, q, x3);
-      store0(sm, AX, x3);
+      store0(sm, aX, x3);
       store0(sm, T, t);
       sync();
     }
     // ZZZ3 = T2 PPP, S1 PPP, R (Q - X3)
-    level<3>(sm, AZZZ, T2, PPP, S1, S1, PPP, T, R, T);
+    level<3>(sm, aZZZ, T2, PPP, S1, S1, PPP, T, R, T);
     {
       uint32_t a[N], b[N], y3[N];
       E::ld(a, at(sm, T));
       E::ld(b, at(sm, S1));
       Fp::sub(y3, a, b);                // Y3 = R(Q - X3) - S1 PPP
-      store0(sm, AY, y3);
+      store0(sm, aY, y3);
       sync();
     }
   }
 
+  // slots base .. base+3 (a point) back to memory (4 lanes)
+  GZ_DEV static void store_pt(uint32_t* dst, uint32_t* sm, int base) {
+    for (int i = lane(); i < 4 * N; i += 4) dst[i] = sm[base * N + i];
+    sync();
+  }
   // A <- the group's sum slots back to memory (4 lanes)
   GZ_DEV static void store_a(uint32_t* dst, uint32_t* sm) {
     for (int i = lane(); i < 4 * N; i += 4) dst[i] = sm[AX * N + i];

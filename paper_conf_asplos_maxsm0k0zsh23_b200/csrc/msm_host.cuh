@@ -644,6 +644,9 @@ struct Impl {
           }
           GZ_CHECK(cudaFuncSetAttribute(k_reduce_bits<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         (int)rb_smem_bytes<C>()));
+          if constexpr (coop_tree<C>())
+            GZ_CHECK(cudaFuncSetAttribute(k_reduce_seg_coop<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                          (int)(32 * CoopS<C>::WORDS * 4)));
           GZ_CHECK(cudaFuncSetAttribute(k_heavy_tree<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                         (int)((size_t)HEAVY_THREADS * 4 * N * 4)));
           return GZKP_SUCCESS;
@@ -753,8 +756,22 @@ struct Impl {
           const int v = e ? atoi(e) : 64;              // measured: 64 / 32 / 128 = 1.02 / 1.03 / 1.05 ms
           return (v >= 32 && v <= 128 && v % 32 == 0) ? v : 64;
         }();
-        k_reduce_seg<C><<<(total + rcta - 1) / rcta, rcta, 0, ss>>>(U(p.o_buckets), U(p.o_offsets), t_lo, gw,
-                                                                    p.B, sb.seg, segT, segR);
+        static const bool seg_coop = [] {
+          const char* e = getenv("GZKP_SEG_COOP");
+          return coop_tree<C>() && (e ? atoi(e) != 0 : true);
+        }();
+        // cooperative chains only where the reduction is small enough to be
+        // latency-bound (round 2: BLS12-381 2^19 prepared, 64K adds, reduce
+        // 0.393 -> 0.288 ms; 1M-add reductions -- standard 2^19 / 2^22,
+        // prepared 2^22, MNT4-753 -- measured 10-12 % slower)
+        if (seg_coop && (uint64_t)gw * p.B * 2 <= 262144) {
+          const unsigned cgrid = (unsigned)((total + 31) / 32);
+          k_reduce_seg_coop<C><<<cgrid, 128, 32 * CoopS<C>::WORDS * 4, ss>>>(U(p.o_buckets), U(p.o_offsets), t_lo,
+                                                                            gw, p.B, sb.seg, segT, segR);
+        } else {
+          k_reduce_seg<C><<<(total + rcta - 1) / rcta, rcta, 0, ss>>>(U(p.o_buckets), U(p.o_offsets), t_lo, gw,
+                                                                      p.B, sb.seg, segT, segR);
+        }
         GZ_CHECK(cudaGetLastError());
         const int NB = ilog2_u64(G);
         const uint32_t nsl = (G + RB_PER - 1) / RB_PER;

@@ -910,6 +910,43 @@ __global__ void __launch_bounds__(128, 2) k_reduce_seg(const uint32_t* __restric
   }
 }
 
+// k_reduce_seg on 4-lane CoopS groups (N >= 12, GZKP_SEG_COOP): a segment's
+// two running sums are one group's chain of cooperative adds -- ~3.5x lower
+// latency per add than one thread at about the same issue cost (a level's
+// four products fill the group's four lanes), so the 2s-add chains stop
+// being latency-bound.  32 groups per 128-thread CTA; dynamic shared memory
+// 32 x CoopS::WORDS words.  Used for small (latency-bound) reductions only:
+// on million-add reductions the group's redundant field additions cost more
+// issue slots than the lower latency saves (msm_host.cuh).
+template <class C>
+__global__ void __launch_bounds__(128) k_reduce_seg_coop(const uint32_t* __restrict__ buckets,
+                                                         const uint32_t* __restrict__ offsets, int t_lo, int W,
+                                                         uint32_t B, int s, uint32_t* __restrict__ segT,
+                                                         uint32_t* __restrict__ segR) {
+  using CS = CoopS<C>;
+  constexpr int N = C::N;
+  extern __shared__ __align__(16) uint32_t seg_smem[];
+  uint32_t* gs = seg_smem + (threadIdx.x >> 2) * CS::WORDS;
+  const uint32_t G = B / s;
+  const uint32_t total = (uint32_t)W * G;
+  const uint32_t gpb = blockDim.x >> 2;
+  for (uint32_t id = blockIdx.x * gpb + (threadIdx.x >> 2); id < total; id += gridDim.x * gpb) {
+    const uint32_t t = t_lo + id / G, g = id % G;
+    CS::set_inf_a(gs, CS::AX);          // R (slots AX..)
+    CS::set_inf_a(gs, CS::CX);          // T (slots CX..)
+    for (int u = s - 1; u >= 0; --u) {
+      const uint32_t key = t * B + g * s + u;
+      if (__ldg(offsets + key + 1) != __ldg(offsets + key)) {
+        CS::put_words(gs, CS::BX, buckets + (size_t)key * 4 * N);
+        CS::add(gs, CS::AX, CS::BX);    // R += B_{gs+u+1}
+      }
+      CS::add(gs, CS::CX, CS::AX);      // T += R
+    }
+    CS::store_pt(segT + (size_t)id * 4 * N, gs, CS::CX);
+    CS::store_pt(segR + (size_t)id * 4 * N, gs, CS::AX);
+  }
+}
+
 constexpr uint32_t RB_PER = 512;          // set elements per k_reduce_bits CTA
 constexpr int RB_THREADS = 128;
 // the serial chains and short trees of the reduction run on CoopS groups for
