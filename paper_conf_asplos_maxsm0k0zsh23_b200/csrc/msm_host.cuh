@@ -43,6 +43,8 @@ struct Plan {
   uint64_t E_max = 0, chunks_max = 0;
   // workspace byte offsets
   size_t o_scc = 0, o_idx = 0, o_ncnt = 0;   // zero-scalar compaction (non-prepared calls)
+  size_t o_ones = 0, o_opart = 0, o_oping = 0;  // the scalar-1 points (k_ones_sum) and their run sums
+  uint32_t ones_runs = 0;
   size_t o_pts = 0, o_codes = 0, o_counts = 0, o_offsets = 0, o_cursor = 0, o_tiles = 0, o_vals = 0,
          o_spay = 0, o_heavy = 0, o_hlist = 0, o_hjobs = 0, o_state = 0, o_buckets = 0, o_seg = 0, o_mid = 0, o_terms = 0, o_hot = 0, o_cb = 0, o_mcnt = 0, o_win = 0, total = 0;
   size_t seg_stride = 0;  // points between segT and segR in o_seg
@@ -332,7 +334,11 @@ struct Impl {
     if (!prepared) {
       p.o_scc = take(n * NS * 4);
       p.o_idx = take(n * 4);
-      p.o_ncnt = take(4 * 8);      // counters [2] + ranges [4]
+      p.o_ncnt = take(4 * 8);      // counters [2] + ranges [4] + ones counter [1]
+      p.ones_runs = (uint32_t)((n + ONES_RUN - 1) / ONES_RUN);
+      p.o_ones = take(n * 4);
+      p.o_opart = take((size_t)p.ones_runs * 4 * N * 4);
+      p.o_oping = take(((size_t)p.ones_runs + TREE_SLICE - 1) / TREE_SLICE * 4 * N * 4);
     }
     p.o_codes = take((size_t)p.W * n * 4);
     p.o_counts = take((size_t)p.M * 4);
@@ -567,6 +573,14 @@ struct Impl {
       return e ? atoi(e) != 0 : false;
     }();
     const bool canon = Canon<C>::ON && canon_env && !call.prepared && !mixed && !minb3 && p.aff_levels == 0;
+    // the scalar-1 points summed apart from the buckets (k_ones_sum; G1
+    // curves up to 12 limbs; GZKP_ONES=0 keeps them in window 0's bucket 1)
+    static const bool ones_env = [] {
+      const char* e = getenv("GZKP_ONES");
+      return e ? atoi(e) != 0 : true;
+    }();
+    const bool ones_on = Canon<C>::ON && N <= 12 && ones_env && !call.prepared && !canon;
+    const uint32_t* ones_total = nullptr;
     // a1: points -> Montgomery (skipped for prepared handles and the canonical hot loop)
     const uint32_t* pts = (const uint32_t*)call.points;
     const uint32_t* sc_sorted = nullptr;
@@ -575,9 +589,10 @@ struct Impl {
     if (!call.prepared) {
       // drop the zero scalars (small ones to the back), then convert the
       // remaining points in the compacted order
-      GZ_CHECK(cudaMemsetAsync(U(p.o_ncnt), 0, 8, s));
+      GZ_CHECK(cudaMemsetAsync(U(p.o_ncnt), 0, 7 * 4, s));
       k_compact<C><<<(unsigned)((n + 255) / 256), 256, 0, s>>>((const uint32_t*)call.scalars, n, p.c, U(p.o_scc),
-                                                              U(p.o_idx), U(p.o_ncnt));
+                                                              U(p.o_idx), U(p.o_ncnt),
+                                                              ones_on ? U(p.o_ones) : nullptr);
       k_compact_ranges<<<1, 1, 0, s>>>(U(p.o_ncnt), (uint32_t)n, U(p.o_ncnt) + 2);
       if (canon) {
         remap = U(p.o_idx);                  // entries name the original point
@@ -591,6 +606,25 @@ struct Impl {
       sc_sorted = U(p.o_scc);
       rng = U(p.o_ncnt) + 2;
       launches += 4;
+      if constexpr (Canon<C>::ON && N <= 12) if (ones_on) {
+        // run sums of the ones, then slice trees level by level (ping-pong)
+        k_ones_sum<C><<<(p.ones_runs + 127) / 128, 128, 0, s>>>((const uint32_t*)call.points, U(p.o_ones),
+                                                               U(p.o_ncnt) + 6, p.ones_runs, U(p.o_opart));
+        uint32_t* src = U(p.o_opart);
+        uint32_t* dst = U(p.o_oping);
+        uint32_t cnt = p.ones_runs, div = 1;
+        ++launches;
+        while (cnt > 1) {
+          const uint32_t nb = (cnt + TREE_SLICE - 1) / TREE_SLICE;
+          k_tree_slices<C><<<nb, 128, 32 * CoopS<C>::WORDS * 4, s>>>(src, cnt, dst, U(p.o_ncnt) + 6, div);
+          cnt = nb;
+          div *= TREE_SLICE;
+          std::swap(src, dst);
+          ++launches;
+        }
+        GZ_CHECK(cudaGetLastError());
+        ones_total = src;
+      }
     }
     // a2 + a3: signed digits, bucket histogram, offsets, sort by bucket
     if (gzkp_status st = sort_stage(call, p, ws, &launches, sc_sorted, rng, remap)) return st;
@@ -785,6 +819,11 @@ struct Impl {
         k_reduce_bits_sum<C><<<gw, 32, 0, ss>>>(U(p.o_terms), NB, U(p.o_win) + (size_t)t_lo * 4 * N);
         GZ_CHECK(cudaGetLastError());
         launches += 4;
+        if constexpr (Canon<C>::ON && N <= 12) if (ones_total && t_lo == 0) {   // W_0 += the ones' sum (weight 1)
+          k_add_point<C><<<1, 32, 0, ss>>>(U(p.o_win), ones_total);
+          GZ_CHECK(cudaGetLastError());
+          ++launches;
+        }
         ev_reduced = profile_event(prof, ss);
         if (ctx) {
           const int evi = 16 + (int)(gi * 8 + k) % 40;

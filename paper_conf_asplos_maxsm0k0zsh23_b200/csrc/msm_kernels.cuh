@@ -112,12 +112,14 @@ __global__ void __launch_bounds__(256) k_to_mont(const uint32_t* __restrict__ in
 // compacted arrays, [n - n_small, n), and the digit and scatter kernels run
 // every window over the "big" range [0, n_big) but only window 0 over the
 // small range.  count[0] = n_big, count[1] = n_small.
+// ones (may be null): the indices of the points whose scalar is exactly 1 go
+// to ones[0 .. count[6]) instead of the small range (k_ones_sum adds them).
 template <class C>
 __global__ void __launch_bounds__(256) k_compact(const uint32_t* __restrict__ sc, size_t n, int c,
                                                  uint32_t* __restrict__ sc_c, uint32_t* __restrict__ idx,
-                                                 uint32_t* __restrict__ count) {
+                                                 uint32_t* __restrict__ count, uint32_t* __restrict__ ones) {
   constexpr int NS = C::NS;
-  __shared__ uint32_t s_warp[8], s_wsm[8], s_base, s_sbase;
+  __shared__ uint32_t s_warp[8], s_wsm[8], s_won[8], s_base, s_sbase, s_obase;
   const size_t i = (size_t)blockIdx.x * 256 + threadIdx.x;
   uint32_t k[NS];
   bool nz = false, small = false;
@@ -141,24 +143,30 @@ __global__ void __launch_bounds__(256) k_compact(const uint32_t* __restrict__ sc
     nz = any != 0;
     small = nz && high == 0 && k[0] < (1u << (c - 1));
   }
-  const bool big = nz && !small;
+  const bool one = ones && small && k[0] == 1u;
+  small = small && !one;
+  const bool big = nz && !small && !one;
   const unsigned m = __ballot_sync(0xffffffffu, big), ms = __ballot_sync(0xffffffffu, small);
+  const unsigned mo = __ballot_sync(0xffffffffu, one);
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  if (lane == 0) { s_warp[w] = __popc(m); s_wsm[w] = __popc(ms); }
+  if (lane == 0) { s_warp[w] = __popc(m); s_wsm[w] = __popc(ms); s_won[w] = __popc(mo); }
   __syncthreads();
   if (threadIdx.x == 0) {
-    uint32_t tot = 0, tots = 0;
+    uint32_t tot = 0, tots = 0, toto = 0;
 #pragma unroll
     for (int q = 0; q < 8; ++q) {
-      const uint32_t cb = s_warp[q], cs = s_wsm[q];
+      const uint32_t cb = s_warp[q], cs = s_wsm[q], co = s_won[q];
       s_warp[q] = tot; tot += cb;
       s_wsm[q] = tots; tots += cs;
+      s_won[q] = toto; toto += co;
     }
     s_base = tot ? atomicAdd(count, tot) : 0u;
     s_sbase = tots ? atomicAdd(count + 1, tots) : 0u;
+    s_obase = toto ? atomicAdd(count + 6, toto) : 0u;
   }
   __syncthreads();
-  if (nz) {
+  if (one) ones[s_obase + s_won[w] + __popc(mo & ((1u << lane) - 1u))] = (uint32_t)i;
+  if (nz && !one) {
     const uint32_t pos = big ? s_base + s_warp[w] + __popc(m & ((1u << lane) - 1u))
                              : (uint32_t)(n - 1 - (s_sbase + s_wsm[w] + __popc(ms & ((1u << lane) - 1u))));
     if constexpr (NS % 4 == 0) {
@@ -625,6 +633,100 @@ struct Canon {
     Fp::mul_sum(A.Y, R, t, PP, PPP);    // Y3 = R(Q - X3) - Y1 PPP
   }
 };
+
+// ---- the sparse witness's ones ("many 0s and 1s"): points
+// whose scalar is exactly 1 skip the bucket pipeline.  k_compact lists them;
+// k_ones_sum adds runs of ONES_RUN of them straight from the caller's
+// canonical points with the primed accumulator of Canon (every thread starts
+// and flushes a run at the same time, so unlike the hot loop no lane waits on
+// another's conversion); k_tree_slices sums the run partials in slices of
+// 512 (CoopS group trees), level by level; k_add_point adds the total to
+// window 0's sum W_0, whose weight is 1.
+constexpr uint32_t ONES_RUN = 64;
+constexpr uint32_t TREE_SLICE = 512;
+template <class C>
+__global__ void __launch_bounds__(128) k_ones_sum(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ ones,
+                                                  const uint32_t* __restrict__ cnt_ptr, uint32_t runs,
+                                                  uint32_t* __restrict__ part) {
+  using Fp = F<C>;
+  using E = EC<C>;
+  constexpr int N = C::N;
+  const uint32_t r = blockIdx.x * blockDim.x + threadIdx.x;
+  const uint32_t cnt = *cnt_ptr;
+  // runs past the live ones are never read (run 0 always writes, O if none)
+  if (r >= runs || (r > 0 && r * ONES_RUN >= cnt)) return;
+  const uint32_t lo = r * ONES_RUN, hi = min(cnt, lo + ONES_RUN);
+  typename E::Xyzz acc;
+  bool inf = true;
+  uint32_t xn[N], yn[N];
+  if (lo < hi) {
+    const size_t i = __ldg(ones + lo);
+    E::ld(xn, pts + i * 2 * N);
+    E::ld(yn, pts + i * 2 * N + N);
+  }
+  for (uint32_t j = lo; j < hi; ++j) {
+    uint32_t x[N], y[N];
+    Fp::copy(x, xn);
+    Fp::copy(y, yn);
+    if (j + 1 < hi) {                   // one point ahead
+      const size_t i = __ldg(ones + j + 1);
+      E::ld(xn, pts + i * 2 * N);
+      E::ld(yn, pts + i * 2 * N + N);
+    }
+    if (Fp::is_zero(x) && Fp::is_zero(y)) continue;   // identity input point
+    if (inf) {
+      Canon<C>::start(acc, x, y);
+      inf = false;
+    } else {
+      Canon<C>::madd(acc, x, y);
+      inf = E::is_inf(acc);
+    }
+  }
+  if (inf) E::set_inf(acc);
+  else Canon<C>::unprime(acc);
+  E::store(part + (size_t)r * 4 * N, acc);
+}
+
+// out[b] = sum of v[b*TREE_SLICE .. min(cnt, (b+1)*TREE_SLICE)) (4N words
+// each); v is overwritten.  128 threads = 32 CoopS groups, dynamic shared
+// memory 32 x CoopS::WORDS words.
+// ones_cnt (device, may be null): only the first ceil(ceil(*ones_cnt /
+// ONES_RUN) / div) elements of v are live (div = TREE_SLICE^level); slices past
+// them write O without work, so a dense input (no ones) costs ~nothing.
+template <class C>
+__global__ void __launch_bounds__(128) k_tree_slices(uint32_t* __restrict__ v, uint32_t cnt,
+                                                     uint32_t* __restrict__ out, const uint32_t* __restrict__ ones_cnt,
+                                                     uint32_t div) {
+  constexpr int N = C::N;
+  extern __shared__ __align__(16) uint32_t tree_smem[];
+  const uint32_t lo = blockIdx.x * TREE_SLICE;
+  if (lo >= cnt) return;                // CTA-uniform
+  if (ones_cnt) {
+    const uint32_t runs = (*ones_cnt + ONES_RUN - 1) / ONES_RUN;
+    cnt = min(cnt, (runs + div - 1) / div);
+    if (lo >= cnt) {                    // no live element in this slice: O
+      typename EC<C>::Xyzz O;
+      EC<C>::set_inf(O);
+      if (threadIdx.x == 0) EC<C>::store(out + (size_t)blockIdx.x * 4 * N, O);
+      return;
+    }
+  }
+  uint32_t* base = v + (size_t)lo * 4 * N;
+  CoopS<C>::tree_sum(base, (int)min(TREE_SLICE, cnt - lo), tree_smem, 32);
+  for (int i = threadIdx.x; i < 4 * N; i += blockDim.x) out[(size_t)blockIdx.x * 4 * N + i] = base[i];
+}
+
+// dst += src (XYZZ, 4N words each) by one CoopS group
+template <class C>
+__global__ void __launch_bounds__(32) k_add_point(uint32_t* __restrict__ dst, const uint32_t* __restrict__ src) {
+  using CS = CoopS<C>;
+  __shared__ __align__(16) uint32_t gsm[CS::WORDS];
+  if (threadIdx.x >= 4) return;
+  CS::put_words(gsm, CS::AX, dst);
+  CS::put_words(gsm, CS::BX, src);
+  CS::add(gsm);
+  CS::store_a(dst, gsm);
+}
 
 // CTAs per SM the hot loop is compiled for (registers: 128 / 168 / 255 per
 // thread).  BN254 fits 3 CTAs in 168 registers; for BLS12-381 forcing 3 CTAs

@@ -10,6 +10,8 @@ because the switches are read once per process:
                        tail of each on its own stream
 * GZKP_AFFINE_LEVELS=L  batch-affine tree levels before the XYZZ loop
                        (affine.cuh experiment; mnt4 and toy curves included)
+* GZKP_ONES=0          the scalar-1 points stay in window 0's bucket 1 (the
+                       default sums them apart, k_ones_sum)
 * GZKP_SEG_COOP=0      one-thread segment chains in the bucket reduction
                        everywhere (the default runs small reductions on CoopS groups)
 * GZKP_CANON=1         the canonical-input hot loop (no Montgomery conversion
@@ -56,7 +58,7 @@ print("VARIANT_OK" if ok else "VARIANT_FAIL")
                                  {"GZKP_REDUCE_GROUPS": "3"}, {"GZKP_REDUCE_GROUPS": "16"},
                                  {"GZKP_REDUCE_GROUPS": "2", "GZKP_PIPELINE": "1"},
                                  {"GZKP_CANON": "1"}, {"GZKP_CANON": "1", "GZKP_PIPELINE": "2"},
-                                 {"GZKP_SEG_COOP": "0"}],
+                                 {"GZKP_SEG_COOP": "0"}, {"GZKP_ONES": "0"}],
                          ids=lambda e: ",".join(f"{k}={v}" for k, v in e.items()))
 def test_variant_parity(env):
     require_cuda()
